@@ -1,0 +1,366 @@
+#!/usr/bin/env python
+"""Benchmark of the hmmsearch filter hot path on B200 (BASELINE.json metric:
+MSV / P7Viterbi / pipeline GCUPS, fraction of the integer-SIMD roofline).
+
+One step = one pass of the whole hot path over the workload:
+MSV over every sequence -> pass flags -> on-device survivor compaction ->
+Viterbi filter (Lazy-F) over the survivors -> (N > 1) NCCL gather of the
+per-sequence results and survivor lists.  Workload (N=1): BASELINE config 3,
+profile M=400 against the Swiss-Prot-shaped DB (550k sequences, mean length
+~360, 0.1% planted homologs).  With N GPUs each rank holds a 550k-sequence
+length-balanced shard of an N x 550k DB (weak scaling).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+Prints ONE JSON line on rank 0.  --impl reference runs the CPU oracle (the
+reference arm of this tier) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MSV / P7Viterbi / pipeline GCUPS at 1/2/4/8 B200; fraction of int-SIMD roofline"
+ALU_LANES_PER_CLK_SM = 64        # measured: VIADDMNMX/VIMNMX3 issue at 64 lanes/clk/SM (profiles/intpeak)
+MSV_ALU_OPS_PER_CELL = 0.75      # VIADDMNMX.S16x2 (1 per 2 cells) + VIMNMX3.S16x2 (1 per 4 cells)
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)),
+            int(os.environ.get("LOCAL_RANK", 0)))
+
+
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in self.rows for n, v in zip(names, r[5:9]) if v.strip().lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def workload(args, world):
+    from paper_conf_ipps_jiangg15_b200 import synth
+    c = dict(synth.CONFIGS[args.config])
+    if isinstance(c["M"], tuple):
+        c["M"], c["pseed"] = c["M"][args.which], c["pseed"][args.which]
+    n_rank = args.nseq or c["N"]
+    prof = synth.make_profile(c["M"], c["pseed"])
+    db = synth.make_db(n_rank * world, c["mu_ln"], c["sigma"], c["dseed"], planted=c["planted"], profile=prof)
+    return c, prof, db
+
+
+# ------------------------------------------------------------------------------------------ reference
+def run_reference(args):
+    """The oracle (reference arm of this tier), timed on the host cores on a bounded
+    sample of the same workload: MSV on every sampled sequence, Viterbi on its MSV survivors."""
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return
+    import oracle
+    c, prof, db = workload(args, 1)
+    oracle.build()
+    mp, vp = oracle.MSVProfile(prof.msc), oracle.VitProfile(prof.msc, prof.tsc)
+    ev = oracle_calibrate(oracle, prof)
+    rng = np.random.default_rng(0)
+    ncores = os.cpu_count() or 1
+    times, cells = [], []
+    for step in range(args.warmup + args.steps):
+        ids = np.sort(rng.choice(db.N, size=args.ref_sample, replace=False))
+        dsq, off = db.materialize(ids)
+        lens = np.diff(off)
+        t0 = time.perf_counter()
+        m = oracle.msv_db(mp, dsq, off, nthreads=ncores)
+        sv = np.array([j for j, (r, L) in enumerate(zip(m, lens))
+                       if oracle.msv_pass(int(r), int(L), ev[0], ev[1], args.F1)], dtype=np.int64)
+        if len(sv):
+            oracle.vit_db(vp, dsq, off, ids=sv, nthreads=ncores)
+        t = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(t)
+            cells.append(c["M"] * int(lens.sum()))
+    v = sum(cells) / sum(times) / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "GCUPS", "n_gpus": 0,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * sum(times) / len(times), 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8/s16",
+            "data": "synthetic",
+            "config": {"workload": "config%d sample" % args.config, "M": c["M"], "sample_seqs": args.ref_sample},
+            "cpu_baseline": {"value": round(v, 4), "unit": "GCUPS", "cores": ncores, "kind": "oracle",
+                             "sample": "%d random sequences per step of the config-%d DB (MSV all, Viterbi on "
+                                       "MSV survivors)" % (args.ref_sample, args.config)},
+            "e2e": {"value": round(v, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def oracle_calibrate(oracle, prof, n=1000, L=200):
+    from paper_conf_ipps_jiangg15_b200 import synth
+    cal = synth.Database(np.full(n, L, np.int32), seed=7)
+    dsq, off = cal.materialize()
+    lam = math.log(2)
+    mb = [oracle.bits(oracle.msv_nats(int(r), L), L) for r in oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off)]
+    vb = [oracle.bits(oracle.vit_nats(int(r), L), L)
+          for r in oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)]
+    return (oracle.fit_mu(np.array(mb), lam), lam, oracle.fit_mu(np.array(vb), lam), lam)
+
+
+def cpu_baseline(prof, dsq, off, ev, F1, M, sample_every):
+    """Oracle as it stands on this box's host cores, on a bounded sample (every k-th sequence)."""
+    import oracle
+    oracle.build()
+    mp, vp = oracle.MSVProfile(prof.msc), oracle.VitProfile(prof.msc, prof.tsc)
+    n = len(off) - 1
+    ids = np.arange(0, n, sample_every, dtype=np.int64)
+    ncores = os.cpu_count() or 1
+    lens = (off[ids + 1] - off[ids])
+    t0 = time.perf_counter()
+    m = oracle.msv_db(mp, dsq, off, ids=ids, nthreads=ncores)
+    sv = np.array([s for s, r, L in zip(ids, m, lens) if oracle.msv_pass(int(r), int(L), ev[0], ev[1], F1)],
+                  dtype=np.int64)
+    if len(sv):
+        oracle.vit_db(vp, dsq, off, ids=sv, nthreads=ncores)
+    t = time.perf_counter() - t0
+    return {"value": round(M * int(lens.sum()) / t / 1e9, 4), "unit": "GCUPS", "cores": ncores, "kind": "oracle",
+            "sample": "every %d-th sequence of rank 0's shard (%d seqs, %d residues): MSV on all, Viterbi on %d "
+                      "MSV survivors; %.1f s" % (sample_every, len(ids), int(lens.sum()), len(sv), t)}
+
+
+# ------------------------------------------------------------------------------------------ main arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="hmg", choices=["hmg", "reference"])
+    ap.add_argument("--config", type=int, default=3)
+    ap.add_argument("--which", type=int, default=0, help="profile index for config 5")
+    ap.add_argument("--nseq", type=int, default=0, help="sequences per rank (default: the config's N)")
+    ap.add_argument("--F1", type=float, default=0.02)
+    ap.add_argument("--F2", type=float, default=1e-3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-sample-every", type=int, default=11)
+    ap.add_argument("--ref-sample", type=int, default=20000)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_jiangg15_b200 import build, hmg
+    from paper_conf_ipps_jiangg15_b200 import dist as hdist
+
+    rank, world, local = env_rank()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if rank == 0:
+        build.build()
+    if world > 1:
+        dist.barrier()
+    hmg.lib()
+
+    c, prof, gdb = workload(args, world)
+    M = c["M"]
+    ids = hdist.snake_shard(gdb.lengths, world, rank)
+    dsq, off = gdb.materialize(ids)
+    ev = hdist.calibrate(prof.msc, prof.tsc, device=local)
+    P = hmg.Profile(prof.msc, prof.tsc, ev=ev, device=local)
+    D = hmg.Database(dsq, off, device=local)
+    n = D.nseq
+    res_local = D.residues
+    out = hmg.alloc_outputs(n, local)
+    gids = torch.as_tensor(ids, device=dev)
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
+
+    def step():
+        hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=stream, **out)
+        if world > 1:
+            packed = hdist.pack_results(out["msv_raw"], out["vit_raw"], out["flags"])
+            hdist.gather(packed, out["survivor_ids"], out["n_survivors"], gids, world)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ---------------------------------------------------------------- timed region (device-resident inputs)
+    hmg.hmg_set_stage_timing(True)
+    launches0 = hmg.hmg_kernel_launches()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    stages = []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            flush.zero_()                              # L2 flush between timed steps (outside the events)
+            evs[i][0].record(stream)
+            step()
+            evs[i][1].record(stream)
+            stages.append(hmg.hmg_stage_times())       # waits for this step's last stage event
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = hmg.hmg_kernel_launches() - launches0
+    hmg.hmg_set_stage_timing(False)
+    ms = [a.elapsed_time(b) for a, b in evs]
+    t_step = sum(ms) / len(ms)
+    t_max = torch.tensor([t_step], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    t_step = float(t_max.item())
+
+    ns = int(out["n_survivors"].item())
+    surv = out["survivor_ids"][:ns].cpu().numpy()
+    surv_res = int(D.lengths[surv].sum()) if ns else 0
+    tot = torch.tensor([res_local, surv_res, ns, n], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot)
+    res_all, surv_all, ns_all, n_all = [float(x) for x in tot.tolist()]
+    cells_all = M * res_all
+    value = cells_all / (t_step * 1e-3) / 1e9
+
+    st = {k: statistics.mean([s[k] for s in stages]) for k in stages[0]}
+    msv_ms, vit_ms = st["msv_kernel"], st["vit_kernel"]
+    msv_gcups = M * res_local / (msv_ms * 1e-3) / 1e9
+    vit_gcups = (M * surv_res / (vit_ms * 1e-3) / 1e9) if vit_ms > 0 else None
+    peaks, src = load_peaks()
+    clock = clk.summary()
+    f_peak = float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    p_int = ALU_LANES_PER_CLK_SM * nsm * f_peak / 1e12                      # T lane-ops/s
+    achieved = MSV_ALU_OPS_PER_CELL * M * res_local / (msv_ms * 1e-3) / 1e12
+    roofline = {"bound": "alu", "kernel": "msv_fast_kernel", "achieved": round(achieved, 3), "peak": round(p_int, 3),
+                "unit": "T int-lane-ops/s", "frac": round(achieved / p_int, 4),
+                "traffic": None, "peak_source": "%s sm_max_mhz x %d SMs x %d lanes/clk (ALU pipe, measured "
+                                                "profiles/intpeak)" % (src, nsm, ALU_LANES_PER_CLK_SM),
+                "algorithmic_ops_per_cell": MSV_ALU_OPS_PER_CELL,
+                "kernel_ms": round(msv_ms, 4), "kernel_share_of_step": round(msv_ms / t_step, 4)}
+
+    # ---------------------------------------------------------------- end to end through the C ABI (host buffers)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        img = torch.empty(D.packed_bytes // 4, dtype=torch.int32, pin_memory=True)
+        D.image(img)
+        h_msv = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        h_vit = torch.empty(n, dtype=torch.int16, pin_memory=True)
+        h_flags = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        h_ns = torch.empty(1, dtype=torch.int64, pin_memory=True)
+        e_ms = []
+        for i in range(args.warmup + args.steps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            D.upload(img, stream=stream)                                   # H2D of the packed DB
+            hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=stream, **out)
+            h_msv.copy_(out["msv_raw"], non_blocking=True)                 # D2H of the results
+            h_vit.copy_(out["vit_raw"], non_blocking=True)
+            h_flags.copy_(out["flags"], non_blocking=True)
+            h_ns.copy_(out["n_survivors"], non_blocking=True)
+            b.record(stream)
+            b.synchronize()
+            if i >= args.warmup:
+                e_ms.append(a.elapsed_time(b))
+        te = sum(e_ms) / len(e_ms)
+        e2e = {"value": round(M * res_local / (te * 1e-3) / 1e9, 3), "unit": "GCUPS",
+               "h2d_bytes_per_step": int(D.packed_bytes), "d2h_bytes_per_step": int(n * 4 + 8),
+               "ms_per_step": round(te, 3)}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(prof, dsq, off, ev, args.F1, M, args.cpu_sample_every)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(t_step, 4), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u8/s16", "data": "synthetic",
+            "config": {"workload": "config%d: M=%d MSV -> on-device compaction -> P7Viterbi (Lazy-F), "
+                                   "Swiss-Prot-shaped DB" % (args.config, M),
+                       "M": M, "nseq_per_rank": n, "residues_per_rank": res_local, "nseq_total": int(n_all),
+                       "residues_total": int(res_all), "F1": args.F1, "F2": args.F2,
+                       "l2": "flushed (256 MiB write) before every timed step, outside its events",
+                       "parallelism": "db-shard x%d (snake length-balanced), NCCL all_gather of results" % world},
+            "stages": {"msv_kernel_ms": round(msv_ms, 4), "msv_gcups": round(msv_gcups, 2),
+                       "msv_redo_ms": round(st["msv_redo"], 4),
+                       "flags_compaction_ms": round(st["msv_flags_compaction"], 4),
+                       "vit_kernel_ms": round(vit_ms, 4), "vit_gcups": round(vit_gcups, 2) if vit_gcups else None,
+                       "vit_flags_ms": round(st["vit_flags"], 4),
+                       "survivors": int(ns_all), "survivor_frac": round(ns_all / max(n_all, 1), 5),
+                       "survivor_residues": int(surv_all)},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches),
+            "clocks": clock,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,193 @@
+/*
+ * hmg.h -- C ABI of the B200 (sm_100a) hmmsearch hot path: HMMER 3.0 MSV filter
+ * and Viterbi filter (P7Viterbi with Lazy-F) scoring one profile HMM against
+ * every sequence of a protein database.
+ *
+ * Paper: Jiang & Ganesan, "Fine-Grained Acceleration of HMMER 3.0 via
+ * Architecture-aware Optimization on Massively Parallel Processors", IPDPSW
+ * 2015.  "P:NNN" cites a line of the paper text.  The problem is
+ * stated at P:21-23 / P:46-53 (score each target sequence against a query
+ * profile, MSV then P7Viterbi, pass sequences by P-value threshold), Alg 1
+ * (MSV) and Alg 2 (P7Viterbi).  Where the paper is
+ * silent the HMMER 3.0 reading in DESIGN.md ("Readings", R1-R35) applies.
+ *
+ * Conventions (all entry points):
+ *   - Plain C, no exceptions; every failure is a status code and leaves no
+ *     side effect (outputs untouched, no handle created).
+ *   - "host" pointers are CPU memory; "device" pointers are CUDA global memory
+ *     on the handle's device.  Ownership of caller buffers never transfers.
+ *   - Compute calls are asynchronous and stream-ordered on `stream`
+ *     (a cudaStream_t passed as void*, NULL = legacy default stream).  They
+ *     return after enqueueing; CUDA launch errors map to HMG_ECUDA.
+ *   - Handles are immutable after creation (internal per-F threshold caches
+ *     are guarded) and may be used from several streams; one handle must not
+ *     be destroyed while work using it is in flight.
+ *   - Sequence indices ("caller order") are positions 0..nseq-1 in the arrays
+ *     given to hmg_db_create.  The DB is internally sorted by length
+ *     (descending) for scheduling; all outputs are in caller order.
+ *   - Overflow is a value, not an error: raw MSV 255 / raw Viterbi 32767 mean
+ *     "score saturated" (+inf nats, P-value 0, always passes; reading R13/R17).
+ *
+ * Residue alphabet (Fig 6): codes 0..28 in the order
+ *   A C D E F G H I K L M N P Q R S T V W Y - B J Z O U X * ~
+ */
+#ifndef HMG_H
+#define HMG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  HMG_OK = 0,
+  HMG_EINVAL = 1,        /* invalid argument (range, NaN, NULL, residue code > 28) */
+  HMG_ENOMEM = 2,        /* host or device allocation failed */
+  HMG_ECUDA = 3,         /* CUDA runtime / launch error (cudaGetLastError cleared) */
+  HMG_EUNSUPPORTED = 4   /* valid but not supported (e.g. no sm_100 device) */
+} hmg_status;
+
+typedef struct hmg_profile hmg_profile; /* quantised profile, host + device tables */
+typedef struct hmg_db hmg_db;           /* packed, length-sorted DB shard on one device */
+
+/* Gumbel parameters of the two filter score distributions, in bits (P:41-45:
+ * Viterbi/MSV high scores are Gumbel with lambda = log 2). */
+typedef struct {
+  double mu_msv, lambda_msv;
+  double mu_vit, lambda_vit;
+} hmg_evparams;
+
+/* Quantised constants (read-only view for tests and score conversion). */
+typedef struct {
+  int M;
+  int bias_b, tbm_b, tec_b, base_b; /* MSV byte system (Alg 1 l.15) */
+  float scale_b;                    /* 3/ln2 (third-bits) */
+  int base_w, xw_e, ddbound_w;      /* Viterbi word system (Alg 2 l.9) */
+  float scale_w;                    /* 500/ln2 */
+  const uint8_t* cost;              /* host [29][M]  biased byte costs, 255 = -inf */
+  const int16_t* rsc;               /* host [29][M]  word emission scores */
+  const int16_t* tsc;               /* host [8][M]   BM MM IM DM MD MI II DD (clamped) */
+  int msv_fast;                     /* 1: exact fast MSV kernel applies (bias < 66 + tbm) */
+  int msv_lanes, msv_regs;          /* MSV kernel geometry: lanes per sequence G, s16x2 regs Q */
+  int vit_lanes, vit_nodes;         /* Viterbi kernel geometry: lanes per sequence, nodes per lane */
+} hmg_quant;
+
+/* ---------------------------------------------------------------- profile */
+
+/* Load and quantise a profile (Alg 1 l.15 P:638; Alg 2 l.15-17 P:687-691).
+ *   M    : model length, 1 <= M <= 100000.
+ *   msc  : host float32 [M][29], match emission log-odds in nats; -INFINITY allowed,
+ *          NaN / +INFINITY rejected.
+ *   tsc  : host float32 [M][8], transition log-probabilities in nats (<= 0 or
+ *          -INFINITY), per node k = 1..M (row k-1):
+ *            0 BM  B->M_k        1 MM  M_{k-1}->M_k   2 IM  I_{k-1}->M_k   3 DM  D_{k-1}->M_k
+ *            4 MD  M_k->D_{k+1}  5 MI  M_k->I_k       6 II  I_k->I_k       7 DD  D_k->D_{k+1}
+ *          Nonexistent transitions (into node 1 from node 0, out of node M) are -INFINITY.
+ *          May be NULL: then only the MSV filter is available.
+ *   ev   : Gumbel parameters for pass flags; may be NULL if no pass flags are requested.
+ *   device : CUDA device ordinal that receives the device tables; device < 0
+ *          makes a host-only handle (quantised tables only; compute calls
+ *          reject it) -- used to inspect the quantiser without a GPU.
+ * Returns HMG_EINVAL on bad M / NaN / +inf / tsc > 0, HMG_ENOMEM, HMG_ECUDA. */
+hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const hmg_evparams* ev,
+                              int device, hmg_profile** out);
+
+/* Fill *out with the quantised constants; the table pointers stay owned by the profile. */
+hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* out);
+
+void hmg_profile_destroy(hmg_profile* p);
+
+/* ---------------------------------------------------------------- database */
+
+/* Pack a database and upload it to `device` (P:417-426 residue packing, Fig 6).
+ *   dsq  : host uint8, all sequences concatenated, codes 0..28.
+ *   off  : host int64 [nseq+1], sequence s is dsq[off[s] .. off[s+1]); lengths >= 1.
+ *   nseq : >= 0.
+ * Sequences are sorted by length (descending, stable), packed 6 residues per
+ * 32-bit word (residue j of a word in bits [5j, 5j+5), bits 30-31 zero, unused
+ * slots 31), each sequence starting on a 16-byte boundary.  device < 0 keeps
+ * the packed image on the host only (inspection without a GPU). */
+hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, int device, hmg_db** out);
+
+int64_t hmg_db_nseq(const hmg_db* db);
+int64_t hmg_db_residues(const hmg_db* db);
+int64_t hmg_db_packed_bytes(const hmg_db* db);   /* size of the packed residue image */
+
+/* Host copy of the schedule: order[j] = caller index of the j-th sequence in
+ * length-descending order (host int32 [nseq]). */
+hmg_status hmg_db_order(const hmg_db* db, int32_t* order);
+
+/* Host copy of the packed residue image (host uint32 [packed_bytes/4]); with
+ * hmg_db_upload it lets a caller keep the image in pinned host memory and
+ * re-send it (end-to-end timing: H2D of the DB inside the timed region). */
+hmg_status hmg_db_image(const hmg_db* db, uint32_t* image);
+
+/* Asynchronously re-upload the packed image (host, ideally pinned) into the DB's
+ * device buffer on `stream`.  The image must come from hmg_db_image of this DB. */
+hmg_status hmg_db_upload(hmg_db* db, const uint32_t* image, void* stream);
+
+void hmg_db_destroy(hmg_db* db);
+
+/* ---------------------------------------------------------------- filters */
+
+/* MSV filter over every sequence (Alg 1).
+ *   raw  : device uint8 [nseq], caller order: raw xJ, 255 = overflow.
+ *   pass : device uint8 [nseq] or NULL: 1 iff P_msv <= F1 (needs ev; F1 in (0, 1]).
+ * HMG_EINVAL if a pass buffer is given without ev, or F1 out of range. */
+hmg_status hmg_msv(const hmg_profile* p, const hmg_db* db, double F1, void* stream, uint8_t* raw,
+                   uint8_t* pass);
+
+/* Viterbi filter (Alg 2; D->D by warp-synchronous Lazy-F) over the
+ * n sequences listed in `ids` (device int32, caller order indices, may repeat).
+ *   raw  : device int16 [nseq]; written only at the listed indices: raw xC,
+ *          32767 = overflow, -32768 = -inf.
+ *   pass : device uint8 [nseq] or NULL: written at the listed indices, 1 iff P_vit <= F2.
+ * ids == NULL means all sequences (n ignored). */
+hmg_status hmg_viterbi(const hmg_profile* p, const hmg_db* db, const int32_t* ids, int64_t n, double F2,
+                       void* stream, int16_t* raw, uint8_t* pass);
+
+/* The hmmsearch filter pipeline (Fig 1): MSV over all sequences ->
+ * pass flags -> on-device stable compaction of survivors -> Viterbi filter over
+ * the survivors only.  All outputs are device buffers in caller order:
+ *   msv_raw      uint8 [nseq]
+ *   vit_raw      int16 [nseq]  (written for survivors only)
+ *   flags        uint8 [nseq]  bit0 MSV pass, bit1 Viterbi pass, bit2 Viterbi was run
+ *   survivor_ids int32 [nseq]  caller indices of MSV survivors, length-descending order
+ *   n_survivors  int64 [1]     device count of survivor_ids
+ * Requires ev and tsc. */
+hmg_status hmg_pipeline(const hmg_profile* p, const hmg_db* db, double F1, double F2, void* stream,
+                        uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                        int64_t* n_survivors);
+
+/* ---------------------------------------------------------------- instrumentation */
+
+/* Number of CUDA kernels this library has launched since it was loaded. */
+int64_t hmg_kernel_launches(void);
+
+/* Stage timing (profiling aid, off by default).  When enabled, hmg_msv /
+ * hmg_viterbi / hmg_pipeline record CUDA events on their stream between
+ * stages; hmg_stage_times waits for the last recorded event and fills
+ * ms[5] with the durations of the most recent call's stages (-1 = not run):
+ *   0 MSV fast kernel   1 MSV exact re-scoring (select + kernel)
+ *   2 MSV pass flags + survivor compaction   3 Viterbi kernel   4 Viterbi flags/scatter
+ * Not thread-safe across concurrent calls (one global set of events). */
+hmg_status hmg_set_stage_timing(int enable);
+hmg_status hmg_stage_times(double* ms);
+
+/* ---------------------------------------------------------------- host helpers (pure) */
+
+/* Raw score -> nats for a length-L target ("Ensure ... (in nats)").
+ * MSV: ((raw - tjb(L)) - 190)/scale_b - 3, +INF for 255.
+ * VF : (raw + move(L) - 12000)/scale_w - 3, +INF for 32767, -INF for -32768. */
+float hmg_msv_nats(int raw, int L);
+float hmg_vit_nats(int raw, int L);
+float hmg_null1_nats(int L);                               /* HMMER null1 (reading R24) */
+double hmg_gumbel_surv(double bits, double mu, double lambda);
+const char* hmg_strerror(hmg_status s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HMG_H */

@@ -1,0 +1,126 @@
+// hmg_internal.h -- private structures of libhmg (host C++ and CUDA sides).
+// Nothing here is shared with oracle/ (the CPU oracle is an independent program).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <mutex>
+#include <vector>
+
+#include "../../include/hmg.h"
+
+namespace hmg {
+
+constexpr int kAlpha = 29;      // 20 + 6 degenerate + 3 gap codes
+constexpr int kRows = 32;       // profile rows in device tables: 29 codes + 3 pad rows (code 31 = pad)
+constexpr int kPadCode = 31;    // unused slots of the last word are 31
+constexpr int kBaseB = 190;     // MSV byte base (reading R1)
+constexpr int kBaseW = 12000;   // Viterbi word base (reading R2)
+constexpr int16_t kNegE = -16384;   // "minus infinity" emission / carry of the s16x2 MSV lanes
+constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
+
+// ---------------------------------------------------------------- MSV kernel arguments
+struct MsvArgs {
+  const uint32_t* words;     // packed residues
+  const uint32_t* woff16;    // [nseq] sorted: word offset / 4 (16-byte units)
+  const int32_t* len;        // [nseq] sorted lengths (descending)
+  int64_t nseq;
+  const uint8_t* tjb;        // [Lmax+1] tjb_b(L)
+  const uint32_t* prof;      // striped s16x2 emission table for (G, Q), kRows rows
+  const uint8_t* cost;       // plain biased costs [kRows][M] (exact kernel)
+  int M, bias, tbm;
+  uint8_t* raw;              // [nseq] sorted order output
+  unsigned long long* counter;  // work-queue counter, zero at launch
+  const int32_t* list;       // exact kernel: sorted indices to redo
+  const int64_t* nlist;      // exact kernel: device count
+  uint8_t* scratch;          // exact kernel: per-warp row buffers
+};
+
+// ---------------------------------------------------------------- Viterbi kernel arguments
+struct VitArgs {
+  const uint32_t* words;
+  const uint32_t* woff16;
+  const int32_t* len;
+  int64_t nseq;
+  const int16_t* move;       // [Lmax+1] move_w(L)
+  const int16_t* rsc;        // register kernel: striped [kRows][G][Q] s16 ; generic: plain [kRows][M]
+  const int32_t* tr;         // register kernel: striped [8][G][Q] s32 ; generic: plain s32 [8][M]
+  int M;
+  const int32_t* list;       // sorted indices to score (NULL = all, in order)
+  const int64_t* nlist;      // device count when list != NULL
+  int16_t* raw_sorted;       // [nseq] output, sorted order
+  unsigned long long* counter;
+  int32_t* scratch;          // generic kernel: per-warp rows
+};
+
+}  // namespace hmg
+
+struct hmg_profile {
+  int M = 0;
+  int device = 0;
+  int bias = 0, tbm = 0, tec = 0, ddbound = -32768;
+  float scale_b = 0.f, scale_w = 0.f;
+  std::vector<uint8_t> cost;  // [29][M]
+  std::vector<int16_t> rsc;   // [29][M]
+  std::vector<int16_t> tsc;   // [8][M] clamped
+  bool has_tsc = false, has_ev = false;
+  hmg_evparams ev{};
+  int msv_fast = 0, msv_G = 0, msv_Q = 0;
+  int vit_G = 0, vit_Q = 0, vit_generic = 0;
+  // device tables
+  uint32_t* d_msv_prof = nullptr;   // striped s16x2 emissions
+  uint8_t* d_cost = nullptr;        // [kRows][M]
+  int16_t* d_rsc = nullptr;         // Viterbi emissions (layout per kernel)
+  int32_t* d_tr = nullptr;          // Viterbi transitions (layout per kernel)
+  size_t msv_prof_bytes = 0, vit_rsc_bytes = 0, vit_tr_bytes = 0;
+  // threshold caches (built on first use per F and DB Lmax)
+  std::mutex mu;
+  struct Thr {
+    double F = -1;
+    int Lmax = -1;
+    void* d = nullptr;
+  } thr_msv, thr_vit;
+};
+
+struct hmg_db {
+  int device = 0;
+  int64_t nseq = 0, residues = 0;
+  int Lmax = 0;
+  int64_t nwords = 0;
+  std::vector<int32_t> order;      // sorted -> caller
+  std::vector<int32_t> len_sorted;
+  uint32_t* d_words = nullptr;
+  uint32_t* d_woff16 = nullptr;
+  int32_t* d_len = nullptr;
+  int32_t* d_order = nullptr;     // sorted -> caller
+  int32_t* d_inv = nullptr;       // caller -> sorted
+  uint8_t* d_tjb = nullptr;       // [Lmax+1]
+  int16_t* d_move = nullptr;      // [Lmax+1]
+  std::vector<uint32_t> host_image;  // host-only handles (device < 0)
+};
+
+namespace hmg {
+extern std::atomic<long long> g_launches;   // kernels launched by libhmg (hmg_kernel_launches)
+// kernels / launchers (CUDA side)
+cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_msv_exact(const MsvArgs& a, int nwarps, cudaStream_t st);
+cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
+int msv_q_max(int G);
+int vit_q_max(int G);
+
+// pipeline helpers (pipeline.cu)
+cudaError_t select_redo(const uint8_t* raw_sorted, int64_t n, int32_t* list, int64_t* count, void* tmp,
+                        cudaStream_t st);
+cudaError_t msv_finish(const uint8_t* raw_sorted, const int32_t* len, const int32_t* order, int64_t n,
+                       const uint16_t* thr, uint8_t* raw_out, uint8_t* pass_out, int32_t* surv_sorted,
+                       int64_t* nsurv, int32_t* surv_caller, void* tmp, cudaStream_t st);
+cudaError_t vit_finish(const int16_t* raw_sorted, const int32_t* list, const int64_t* nlist, int64_t nmax,
+                       const int32_t* len, const int32_t* order, const int32_t* thr, int16_t* raw_out,
+                       uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st);
+cudaError_t to_sorted_ids(const int32_t* caller_ids, int64_t n, const int32_t* inv_order, int32_t* sorted_ids,
+                          cudaStream_t st);
+cudaError_t set_count(int64_t* d, int64_t v, cudaStream_t st);
+size_t scan_tmp_bytes(int64_t n);
+}  // namespace hmg

@@ -1,0 +1,880 @@
+// host.cu -- libhmg host side: quantiser, DB packer/sorter, threshold tables,
+// kernel geometry policy and the C ABI declared in include/hmg.h.
+//
+// The quantiser implements HMMER 3.0's byte and word score systems (the
+// paper: "8-bit saturating scoring system"; "bias", Alg 1 l.15
+// P:638; "-32768" word -inf, Alg 2 l.9 P:674; constants per DESIGN.md R1-R10).
+// It is written independently of oracle/ (no shared code); tests require the
+// two to agree byte-for-byte.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <numeric>
+#include <vector>
+
+#include "hmg_internal.h"
+
+using namespace hmg;
+
+std::atomic<long long> hmg::g_launches{0};
+
+namespace {
+
+// ---------------------------------------------------------------- stage timing (profiling aid)
+// Stages: 0 MSV fast kernel | 1 MSV exact redo (select + kernel) | 2 MSV flags + compaction |
+//         3 Viterbi kernel | 4 Viterbi flags/scatter.  Marks are CUDA events on the call's stream.
+constexpr int kStages = 5;
+struct StageTimer {
+  bool on = false;
+  int device = -1;
+  cudaEvent_t ev[kStages + 1] = {};
+  bool rec[kStages + 1] = {};
+} g_timer;
+std::mutex g_timer_mu;
+
+void mark(int i, cudaStream_t st) {
+  if (!g_timer.on) return;
+  if (cudaEventRecord(g_timer.ev[i], st) == cudaSuccess) g_timer.rec[i] = true;
+}
+void mark_reset() {
+  if (!g_timer.on) return;
+  for (bool& r : g_timer.rec) r = false;
+}
+
+constexpr double kLn2 = 0.693147180559945309417232121458176568;
+
+// ---------------------------------------------------------------- quantisation
+struct Scales {
+  float b = (float)(3.0 / kLn2);    // third-bits (R1)
+  float w = (float)(500.0 / kLn2);  // 1/500 bits (R2)
+};
+
+// unbiased byte cost of a non-positive score, capped at 255 (R3)
+int cost_unbiased(float sc, const Scales& S) {
+  const float c = -roundf(S.b * sc);
+  return c > 255.0f ? 255 : (int)c;
+}
+
+// biased byte cost; 255 is -inf (R4)
+uint8_t cost_biased(float sc, int bias, const Scales& S) {
+  const float c = -roundf(S.b * sc);
+  if (c > (float)(255 - bias)) return 255;
+  const int v = (int)c + bias;
+  return (uint8_t)(v < 0 ? 0 : v);
+}
+
+// word score clamped to int16 (R5)
+int16_t word(float sc, const Scales& S) {
+  const float r = roundf(S.w * sc);
+  if (r >= 32767.0f) return 32767;
+  if (r <= -32768.0f) return -32768;
+  return (int16_t)r;
+}
+
+int tjb_of(int L) { return cost_unbiased(logf(3.0f / (float)(L + 3)), Scales()); }  // R10
+int16_t move_of(int L) { return word(logf(3.0f / (float)(L + 3)), Scales()); }      // R10
+
+// ---------------------------------------------------------------- statistics (R11, R24, R25)
+float msv_nats_of(int raw, int L) {
+  if (raw == 255) return INFINITY;
+  const Scales S;
+  float v = (float)(raw - tjb_of(L)) - (float)kBaseB;
+  v /= S.b;
+  v -= 3.0;
+  return v;
+}
+
+float vit_nats_of(int raw, int L) {
+  if (raw == 32767) return INFINITY;
+  if (raw == -32768) return -INFINITY;
+  const Scales S;
+  float v = (float)(raw + move_of(L)) - (float)kBaseW;
+  v /= S.w;
+  v -= 3.0;
+  return v;
+}
+
+float null1_of(int L) {
+  const float p1 = (float)L / (float)(L + 1);
+  return (float)((float)L * log((double)p1) + log(1.0 - (double)p1));
+}
+
+double gumbel_surv(double x, double mu, double lambda) {
+  const double y = lambda * (x - mu);
+  const double ey = -exp(-y);
+  return fabs(ey) < 5e-9 ? -ey : 1.0 - exp(ey);
+}
+
+bool passes(float nats, int L, double mu, double lambda, double F) {
+  double P;
+  if (nats == INFINITY) P = 0.0;
+  else if (nats == -INFINITY) P = 1.0;
+  else P = gumbel_surv((double)(nats - null1_of(L)) / kLn2, mu, lambda);
+  return !(P > F);
+}
+
+// least raw in [lo, hi] that passes (pass is monotone in raw), hi+1 if none
+template <class Pass>
+int least_passing(int lo, int hi, Pass pass) {
+  if (!pass(hi)) return hi + 1;
+  while (lo < hi) {
+    const int mid = lo + (hi - lo) / 2;
+    if (pass(mid)) hi = mid;
+    else lo = mid + 1;
+  }
+  return lo;
+}
+
+// ---------------------------------------------------------------- helpers
+struct Dev {
+  int saved = -1;
+  explicit Dev(int d) {
+    cudaGetDevice(&saved);
+    if (saved != d) cudaSetDevice(d);
+  }
+  ~Dev() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (saved >= 0 && cur != saved) cudaSetDevice(saved);
+  }
+};
+
+hmg_status cuda_status(cudaError_t e) {
+  if (e == cudaSuccess) return HMG_OK;
+  cudaGetLastError();
+  return e == cudaErrorMemoryAllocation ? HMG_ENOMEM : HMG_ECUDA;
+}
+
+template <class T>
+hmg_status upload(T** d, const T* h, size_t n) {
+  *d = nullptr;
+  if (n == 0) n = 1;
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(d), n * sizeof(T));
+  if (e != cudaSuccess) return cuda_status(e);
+  if (h) e = cudaMemcpy(*d, h, n * sizeof(T), cudaMemcpyHostToDevice);
+  return cuda_status(e);
+}
+
+int env_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return v ? atoi(v) : dflt;
+}
+
+// ---------------------------------------------------------------- kernel geometry
+void msv_geometry(int M, int* G, int* Q) {
+  int g = M <= 128 ? 4 : M <= 512 ? 8 : M <= 1024 ? 16 : 32;
+  const int o = env_int("HMG_MSV_G", 0);
+  if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
+  // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
+  // fast kernel records each cell's value in the cell it feeds (t_{i+1}[k+1]).
+  int q = (M + 2 * g) / (2 * g);
+  while (q > msv_q_max(g) && g < 32) {
+    g *= 2;
+    q = (M + 2 * g) / (2 * g);
+  }
+  *G = g;
+  *Q = q <= msv_q_max(g) ? q : 0;   // 0: no register kernel, exact kernel only
+}
+
+void vit_geometry(int M, int* G, int* Q) {
+  int g = M <= 128 ? 8 : M <= 256 ? 16 : 32;
+  const int o = env_int("HMG_VIT_G", 0);
+  if (o == 8 || o == 16 || o == 32) g = o;
+  int q = (M + g - 1) / g;
+  while (q > vit_q_max(g) && g < 32) {
+    g *= 2;
+    q = (M + g - 1) / g;
+  }
+  *G = g;
+  *Q = q <= vit_q_max(g) ? q : 0;
+}
+
+// striped MSV table: row x, register q of lane z holds e for nodes z*Q+q+1 (lo), (z+G)*Q+q+1 (hi)
+std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
+  const int M = p.M;
+  const int ROWW = Q * G;
+  std::vector<uint32_t> t((size_t)kRows * ROWW);
+  const int n4 = Q / 4, r = Q % 4;
+  auto word_index = [&](int z, int q) {
+    if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
+    int b = n4 * 4 * G;
+    int qq = q - n4 * 4;
+    if (r >= 2) {
+      if (qq < 2) return b + z * 2 + qq;
+      b += 2 * G;
+      qq -= 2;
+    }
+    return b + z;
+  };
+  auto e_of = [&](int x, int node) -> int16_t {   // node 1-based
+    if (x >= kAlpha || node > M) return kNegE;
+    return (int16_t)(p.bias - (int)p.cost[(size_t)x * M + (node - 1)]);
+  };
+  for (int x = 0; x < kRows; ++x)
+    for (int z = 0; z < G; ++z)
+      for (int q = 0; q < Q; ++q) {
+        const uint16_t lo = (uint16_t)e_of(x, z * Q + q + 1);
+        const uint16_t hi = (uint16_t)e_of(x, (z + G) * Q + q + 1);
+        t[(size_t)x * ROWW + word_index(z, q)] = (uint32_t)lo | ((uint32_t)hi << 16);
+      }
+  return t;
+}
+
+// Viterbi register-kernel tables: emissions as s16 pairs in the MSV chunk layout over Q2 words,
+// transitions as s32 [8][G*Q] with node (z*Q+q+1) at z*Q+q; nodes > M are -inf.
+void vit_tables(const hmg_profile& p, int G, int Q, std::vector<uint32_t>* rsc, std::vector<int32_t>* tr) {
+  const int M = p.M;
+  const int Q2 = (Q + 1) / 2;
+  const int ROWW = Q2 * G;
+  rsc->assign(((size_t)kRows * ROWW + 3) / 4 * 4, 0);
+  const int n4 = Q2 / 4, r = Q2 % 4;
+  auto word_index = [&](int z, int q) {
+    if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
+    int b = n4 * 4 * G;
+    int qq = q - n4 * 4;
+    if (r >= 2) {
+      if (qq < 2) return b + z * 2 + qq;
+      b += 2 * G;
+      qq -= 2;
+    }
+    return b + z;
+  };
+  auto r_of = [&](int x, int node) -> int16_t {
+    if (x >= kAlpha || node > M) return (int16_t)kNegW;
+    return p.rsc[(size_t)x * M + node - 1];
+  };
+  for (int x = 0; x < kRows; ++x)
+    for (int z = 0; z < G; ++z)
+      for (int h = 0; h < Q2; ++h) {
+        const uint16_t lo = (uint16_t)r_of(x, z * Q + 2 * h + 1);
+        const uint16_t hi = (2 * h + 1 < Q) ? (uint16_t)r_of(x, z * Q + 2 * h + 2) : (uint16_t)kNegW;
+        (*rsc)[(size_t)x * ROWW + word_index(z, h)] = (uint32_t)lo | ((uint32_t)hi << 16);
+      }
+  tr->assign((size_t)8 * G * Q, kNegW);
+  for (int t = 0; t < 8; ++t)
+    for (int o = 0; o < G * Q; ++o)
+      if (o < M) (*tr)[(size_t)t * G * Q + o] = p.tsc[(size_t)t * M + o];
+}
+
+struct Scratch {
+  std::vector<void*> bufs;
+  cudaStream_t st;
+  explicit Scratch(cudaStream_t s) : st(s) {}
+  void* get(size_t n, cudaError_t* err) {
+    void* p = nullptr;
+    cudaError_t e = cudaMallocAsync(&p, n ? n : 16, st);
+    if (e != cudaSuccess) {
+      *err = e;
+      return nullptr;
+    }
+    bufs.push_back(p);
+    return p;
+  }
+  ~Scratch() {
+    for (void* p : bufs) cudaFreeAsync(p, st);
+  }
+};
+
+// threshold tables, cached per (F, Lmax) in the profile
+hmg_status msv_thr_table(hmg_profile* p, const hmg_db* db, double F, const uint16_t** out) {
+  std::lock_guard<std::mutex> g(p->mu);
+  auto& c = p->thr_msv;
+  if (c.d && c.F == F && c.Lmax >= db->Lmax) {
+    *out = (const uint16_t*)c.d;
+    return HMG_OK;
+  }
+  std::vector<uint16_t> h((size_t)db->Lmax + 1, 256);
+  const double mu = p->ev.mu_msv, lam = p->ev.lambda_msv;
+  for (int L = 1; L <= db->Lmax; ++L)
+    h[L] = (uint16_t)least_passing(0, 254, [&](int r) { return passes(msv_nats_of(r, L), L, mu, lam, F); });
+  if (c.d) cudaFree(c.d);
+  c.d = nullptr;
+  uint16_t* d = nullptr;
+  hmg_status s = upload(&d, h.data(), h.size());
+  if (s != HMG_OK) return s;
+  c.d = d;
+  c.F = F;
+  c.Lmax = db->Lmax;
+  *out = d;
+  return HMG_OK;
+}
+
+hmg_status vit_thr_table(hmg_profile* p, const hmg_db* db, double F, const int32_t** out) {
+  std::lock_guard<std::mutex> g(p->mu);
+  auto& c = p->thr_vit;
+  if (c.d && c.F == F && c.Lmax >= db->Lmax) {
+    *out = (const int32_t*)c.d;
+    return HMG_OK;
+  }
+  std::vector<int32_t> h((size_t)db->Lmax + 1, 32767);
+  const double mu = p->ev.mu_vit, lam = p->ev.lambda_vit;
+  for (int L = 1; L <= db->Lmax; ++L)
+    h[L] = least_passing(-32768, 32766, [&](int r) { return passes(vit_nats_of(r, L), L, mu, lam, F); });
+  if (c.d) cudaFree(c.d);
+  c.d = nullptr;
+  int32_t* d = nullptr;
+  hmg_status s = upload(&d, h.data(), h.size());
+  if (s != HMG_OK) return s;
+  c.d = d;
+  c.F = F;
+  c.Lmax = db->Lmax;
+  *out = d;
+  return HMG_OK;
+}
+
+MsvArgs msv_args(const hmg_profile* p, const hmg_db* db) {
+  MsvArgs a{};
+  a.words = db->d_words;
+  a.woff16 = db->d_woff16;
+  a.len = db->d_len;
+  a.nseq = db->nseq;
+  a.tjb = db->d_tjb;
+  a.prof = p->d_msv_prof;
+  a.cost = p->d_cost;
+  a.M = p->M;
+  a.bias = p->bias;
+  a.tbm = p->tbm;
+  return a;
+}
+
+// MSV over the whole DB into raw_sorted (device, sorted order); fast kernel + exact redo.
+hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
+  cudaError_t e = cudaSuccess;
+  const int64_t n = db->nseq;
+  MsvArgs a = msv_args(p, db);
+  a.raw = raw_sorted;
+  auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+  if (e) return cuda_status(e);
+  if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+  a.counter = ctr;
+  const int nwarps_exact = 148 * 16;
+  if (p->msv_fast && p->msv_Q > 0) {
+    int ok = 0;
+    mark(0, st);
+    if ((e = launch_msv_fast(p->msv_G, p->msv_Q, a, st, &ok))) return cuda_status(e);
+    if (!ok) return HMG_EUNSUPPORTED;
+    mark(1, st);
+    // sequences whose every cell stayed <= B' are rescored exactly (rare)
+    auto* list = (int32_t*)S.get(sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1), &e);
+    auto* cnt = (int64_t*)S.get(sizeof(int64_t), &e);
+    void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
+    auto* scr = (uint8_t*)S.get((size_t)nwarps_exact * 2 * (p->M + 1), &e);
+    if (e) return cuda_status(e);
+    if ((e = select_redo(raw_sorted, n, list, cnt, tmp, st))) return cuda_status(e);
+    a.list = list;
+    a.nlist = cnt;
+    a.scratch = scr;
+    if ((e = launch_msv_exact(a, nwarps_exact, st))) return cuda_status(e);
+    mark(2, st);
+  } else {
+    auto* scr = (uint8_t*)S.get((size_t)nwarps_exact * 2 * (p->M + 1), &e);
+    if (e) return cuda_status(e);
+    a.list = nullptr;
+    a.scratch = scr;
+    mark(0, st);
+    if (n > 0 && (e = launch_msv_exact(a, nwarps_exact, st))) return cuda_status(e);
+    mark(1, st);
+    mark(2, st);
+  }
+  return HMG_OK;
+}
+
+// Viterbi over sorted-order ids (list, device count) into raw_sorted.
+hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
+                   cudaStream_t st, int16_t* raw_sorted, Scratch& S) {
+  cudaError_t e = cudaSuccess;
+  VitArgs a{};
+  a.words = db->d_words;
+  a.woff16 = db->d_woff16;
+  a.len = db->d_len;
+  a.nseq = db->nseq;
+  a.move = db->d_move;
+  a.rsc = p->d_rsc;
+  a.tr = p->d_tr;
+  a.M = p->M;
+  a.list = list;
+  a.nlist = nlist;
+  a.raw_sorted = raw_sorted;
+  auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
+  if (e) return cuda_status(e);
+  if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
+  a.counter = ctr;
+  mark(3, st);
+  if (!p->vit_generic) {
+    int ok = 0;
+    if ((e = launch_vit_reg(p->vit_G, p->vit_Q, a, st, &ok))) return cuda_status(e);
+    if (!ok) return HMG_EUNSUPPORTED;
+  } else {
+    const int nwarps = 148 * 16;
+    auto* scr = (int32_t*)S.get((size_t)nwarps * 6 * (p->M + 1) * sizeof(int32_t), &e);
+    if (e) return cuda_status(e);
+    a.scratch = scr;
+    if ((e = launch_vit_generic(a, nwarps, st))) return cuda_status(e);
+  }
+  mark(4, st);
+  return HMG_OK;
+}
+
+bool bad_float(float v, bool allow_pos) {
+  if (std::isnan(v)) return true;
+  if (v == INFINITY) return true;
+  if (!allow_pos && v > 0.0f) return true;
+  return false;
+}
+
+}  // namespace
+
+// =====================================================================================
+extern "C" {
+
+const char* hmg_strerror(hmg_status s) {
+  switch (s) {
+    case HMG_OK: return "ok";
+    case HMG_EINVAL: return "invalid argument";
+    case HMG_ENOMEM: return "out of memory";
+    case HMG_ECUDA: return "CUDA error";
+    case HMG_EUNSUPPORTED: return "unsupported";
+  }
+  return "unknown status";
+}
+
+int64_t hmg_kernel_launches(void) { return g_launches.load(); }
+
+hmg_status hmg_set_stage_timing(int enable) {
+  std::lock_guard<std::mutex> g(g_timer_mu);
+  if (enable && !g_timer.on) {
+    cudaGetDevice(&g_timer.device);
+    for (auto& e : g_timer.ev)
+      if (cudaEventCreate(&e) != cudaSuccess) return cuda_status(cudaGetLastError());
+    g_timer.on = true;
+  } else if (!enable && g_timer.on) {
+    for (auto& e : g_timer.ev) cudaEventDestroy(e);
+    g_timer = StageTimer();
+  }
+  return HMG_OK;
+}
+
+hmg_status hmg_stage_times(double* ms) {
+  if (!ms) return HMG_EINVAL;
+  std::lock_guard<std::mutex> g(g_timer_mu);
+  if (!g_timer.on) return HMG_EINVAL;
+  for (int i = 0; i < kStages; ++i) ms[i] = -1.0;
+  int last = -1;
+  for (int i = kStages; i >= 0; --i)
+    if (g_timer.rec[i]) { last = i; break; }
+  if (last < 0) return HMG_OK;
+  if (cudaEventSynchronize(g_timer.ev[last]) != cudaSuccess) return cuda_status(cudaGetLastError());
+  for (int i = 0; i < kStages; ++i) {
+    if (!g_timer.rec[i] || !g_timer.rec[i + 1]) continue;
+    float t = 0.f;
+    if (cudaEventElapsedTime(&t, g_timer.ev[i], g_timer.ev[i + 1]) == cudaSuccess) ms[i] = t;
+    else cudaGetLastError();
+  }
+  return HMG_OK;
+}
+
+float hmg_msv_nats(int raw, int L) { return msv_nats_of(raw, L); }
+float hmg_vit_nats(int raw, int L) { return vit_nats_of(raw, L); }
+float hmg_null1_nats(int L) { return null1_of(L); }
+double hmg_gumbel_surv(double bits, double mu, double lambda) { return gumbel_surv(bits, mu, lambda); }
+
+hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const hmg_evparams* ev, int device,
+                              hmg_profile** out) {
+  if (!out || !msc || M < 1 || M > 100000) return HMG_EINVAL;
+  *out = nullptr;
+  for (size_t i = 0; i < (size_t)M * kAlpha; ++i)
+    if (bad_float(msc[i], true)) return HMG_EINVAL;
+  if (tsc)
+    for (size_t i = 0; i < (size_t)M * 8; ++i)
+      if (bad_float(tsc[i], false)) return HMG_EINVAL;
+  if (ev && (!(ev->lambda_msv > 0) || !(ev->lambda_vit > 0) || std::isnan(ev->mu_msv) || std::isnan(ev->mu_vit)))
+    return HMG_EINVAL;
+  if (device >= 0) {   // device < 0: host-only handle (quantised tables, no device copies)
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device >= ndev) {
+      cudaGetLastError();
+      return ndev == 0 ? HMG_EUNSUPPORTED : HMG_EINVAL;
+    }
+  }
+  hmg_profile* p = new (std::nothrow) hmg_profile();
+  if (!p) return HMG_ENOMEM;
+  p->M = M;
+  p->device = device;
+  const Scales S;
+  p->scale_b = S.b;
+  p->scale_w = S.w;
+  // ---- byte profile (R1, R3, R4, R7)
+  float best = 0.0f;
+  for (int k = 0; k < M; ++k)
+    for (int x = 0; x < 20; ++x) best = std::max(best, msc[(size_t)k * kAlpha + x]);
+  p->bias = cost_unbiased(-best, S);
+  p->tbm = cost_unbiased(logf(2.0f / ((float)M * (float)(M + 1))), S);
+  p->tec = cost_unbiased(logf(0.5f), S);
+  p->cost.resize((size_t)kAlpha * M);
+  for (int x = 0; x < kAlpha; ++x)
+    for (int k = 0; k < M; ++k) p->cost[(size_t)x * M + k] = cost_biased(msc[(size_t)k * kAlpha + x], p->bias, S);
+  // ---- word profile (R2, R5, R6)
+  p->rsc.resize((size_t)kAlpha * M);
+  for (int x = 0; x < kAlpha; ++x)
+    for (int k = 0; k < M; ++k) p->rsc[(size_t)x * M + k] = word(msc[(size_t)k * kAlpha + x], S);
+  p->has_tsc = tsc != nullptr;
+  if (tsc) {
+    p->tsc.resize((size_t)8 * M);
+    for (int t = 0; t < 8; ++t)
+      for (int k = 0; k < M; ++k) {
+        int v = word(tsc[(size_t)k * 8 + t], S);
+        const int cap = t == 6 ? -1 : (t == 7 ? 32767 : 0);
+        p->tsc[(size_t)t * M + k] = (int16_t)std::min(v, cap);
+      }
+    int ddb = -32768;
+    for (int k = 2; k <= M - 2; ++k) {
+      const int v = (int)word(tsc[(size_t)(k - 1) * 8 + 7], S) + (int)word(tsc[(size_t)(k + 1) * 8 + 3], S) -
+                    (int)word(tsc[(size_t)(k + 1) * 8 + 0], S);
+      ddb = std::max(ddb, v);
+    }
+    p->ddbound = ddb;
+  }
+  if (ev) {
+    p->has_ev = true;
+    p->ev = *ev;
+  }
+  // ---- kernel geometry and device tables
+  p->msv_fast = p->bias < 66 + p->tbm;   // precondition of the fast MSV kernel
+  msv_geometry(M, &p->msv_G, &p->msv_Q);
+  if (tsc) {
+    vit_geometry(M, &p->vit_G, &p->vit_Q);
+    p->vit_generic = p->vit_Q == 0 || env_int("HMG_VIT_GENERIC", 0);
+  }
+  if (device < 0) {
+    *out = p;
+    return HMG_OK;
+  }
+  Dev dg(device);
+  hmg_status st = HMG_OK;
+  {
+    std::vector<uint8_t> c((size_t)kRows * M, 255);
+    std::copy(p->cost.begin(), p->cost.end(), c.begin());
+    st = upload(&p->d_cost, c.data(), c.size());
+  }
+  if (st == HMG_OK && p->msv_Q > 0) {
+    auto t = msv_table(*p, p->msv_G, p->msv_Q);
+    p->msv_prof_bytes = t.size() * 4;
+    st = upload(&p->d_msv_prof, t.data(), t.size());
+  }
+  if (st == HMG_OK && tsc) {
+    if (!p->vit_generic) {
+      std::vector<uint32_t> r;
+      std::vector<int32_t> t;
+      vit_tables(*p, p->vit_G, p->vit_Q, &r, &t);
+      p->vit_rsc_bytes = r.size() * 4;
+      p->vit_tr_bytes = t.size() * 4;
+      st = upload(reinterpret_cast<uint32_t**>(&p->d_rsc), r.data(), r.size());
+      if (st == HMG_OK) st = upload(&p->d_tr, t.data(), t.size());
+    } else {
+      std::vector<int16_t> r((size_t)kRows * M, (int16_t)kNegW);
+      std::copy(p->rsc.begin(), p->rsc.end(), r.begin());
+      std::vector<int32_t> t(p->tsc.begin(), p->tsc.end());
+      st = upload(&p->d_rsc, r.data(), r.size());
+      if (st == HMG_OK) st = upload(&p->d_tr, t.data(), t.size());
+    }
+  }
+  if (st != HMG_OK) {
+    hmg_profile_destroy(p);
+    return st;
+  }
+  *out = p;
+  return HMG_OK;
+}
+
+hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
+  if (!p || !q) return HMG_EINVAL;
+  q->M = p->M;
+  q->bias_b = p->bias;
+  q->tbm_b = p->tbm;
+  q->tec_b = p->tec;
+  q->base_b = kBaseB;
+  q->scale_b = p->scale_b;
+  q->base_w = kBaseW;
+  q->xw_e = word(logf(0.5f), Scales());
+  q->ddbound_w = p->ddbound;
+  q->scale_w = p->scale_w;
+  q->cost = p->cost.data();
+  q->rsc = p->rsc.data();
+  q->tsc = p->has_tsc ? p->tsc.data() : nullptr;
+  q->msv_fast = p->msv_fast;
+  q->msv_lanes = p->msv_G;
+  q->msv_regs = p->msv_Q;
+  q->vit_lanes = p->vit_generic ? 32 : p->vit_G;
+  q->vit_nodes = p->vit_generic ? 0 : p->vit_Q;
+  return HMG_OK;
+}
+
+void hmg_profile_destroy(hmg_profile* p) {
+  if (!p) return;
+  if (p->device >= 0) {
+    Dev dg(p->device);
+    cudaFree(p->d_msv_prof);
+    cudaFree(p->d_cost);
+    cudaFree(p->d_rsc);
+    cudaFree(p->d_tr);
+    cudaFree(p->thr_msv.d);
+    cudaFree(p->thr_vit.d);
+    cudaGetLastError();
+  }
+  delete p;
+}
+
+hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, int device, hmg_db** out) {
+  if (!out || nseq < 0 || (nseq > 0 && (!dsq || !off)) || nseq > 0x7fffffff) return HMG_EINVAL;
+  *out = nullptr;
+  if (device >= 0) {   // device < 0: host-only handle (packed image kept on the host)
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device >= ndev) {
+      cudaGetLastError();
+      return ndev == 0 ? HMG_EUNSUPPORTED : HMG_EINVAL;
+    }
+  }
+  // validate (codes 0..28; lengths >= 1)
+  int64_t res = 0;
+  int Lmax = 0;
+  for (int64_t s = 0; s < nseq; ++s) {
+    const int64_t L = off[s + 1] - off[s];
+    if (L < 1 || L > 0x3fffffff || off[s] < 0) return HMG_EINVAL;
+    Lmax = std::max<int64_t>(Lmax, L);
+    res += L;
+  }
+  for (int64_t i = 0; i < (nseq ? off[nseq] - off[0] : 0); ++i)
+    if (dsq[off[0] + i] > 28) return HMG_EINVAL;
+  hmg_db* db = new (std::nothrow) hmg_db();
+  if (!db) return HMG_ENOMEM;
+  db->device = device;
+  db->nseq = nseq;
+  db->residues = res;
+  db->Lmax = Lmax;
+  // length sort, descending, stable (schedule order)
+  db->order.resize(nseq);
+  std::iota(db->order.begin(), db->order.end(), 0);
+  std::stable_sort(db->order.begin(), db->order.end(), [&](int32_t a, int32_t b) {
+    return off[a + 1] - off[a] > off[b + 1] - off[b];
+  });
+  db->len_sorted.resize(nseq);
+  std::vector<uint32_t> woff16(nseq);
+  int64_t words = 0;
+  for (int64_t j = 0; j < nseq; ++j) {
+    const int32_t s = db->order[j];
+    const int L = (int)(off[s + 1] - off[s]);
+    db->len_sorted[j] = L;
+    if (words / 4 > 0xffffffffLL) {
+      delete db;
+      return HMG_EUNSUPPORTED;
+    }
+    woff16[j] = (uint32_t)(words / 4);
+    words += ((L + 5) / 6 + 3) / 4 * 4;   // 16-byte aligned runs
+  }
+  db->nwords = words;
+  // pack 6 residues per word, residue j in bits [5j, 5j+5), pad 31 (Fig 6)
+  std::vector<uint32_t> img((size_t)std::max<int64_t>(words, 4), 0xffffffffu);
+  for (int64_t j = 0; j < nseq; ++j) {
+    const int32_t s = db->order[j];
+    const uint8_t* d = dsq + off[s];
+    const int L = db->len_sorted[j];
+    uint32_t* w = img.data() + (size_t)woff16[j] * 4;
+    const int nw = (L + 5) / 6;
+    for (int i = 0; i < nw; ++i) {
+      uint32_t v = 0;
+      for (int b = 0; b < 6; ++b) {
+        const int r = 6 * i + b;
+        v |= (uint32_t)(r < L ? d[r] : kPadCode) << (5 * b);
+      }
+      w[i] = v & 0x3fffffffu;
+    }
+  }
+  std::vector<uint8_t> tjb((size_t)Lmax + 1, 0);
+  std::vector<int16_t> mv((size_t)Lmax + 1, 0);
+  for (int L = 1; L <= Lmax; ++L) {
+    tjb[L] = (uint8_t)tjb_of(L);
+    mv[L] = move_of(L);
+  }
+  std::vector<int32_t> inv(nseq);
+  for (int64_t j = 0; j < nseq; ++j) inv[db->order[j]] = (int32_t)j;
+  if (device < 0) {
+    db->host_image = std::move(img);
+    *out = db;
+    return HMG_OK;
+  }
+  Dev dg(device);
+  hmg_status st = upload(&db->d_words, img.data(), img.size());
+  if (st == HMG_OK) st = upload(&db->d_woff16, woff16.data(), woff16.size());
+  if (st == HMG_OK) st = upload(&db->d_len, db->len_sorted.data(), db->len_sorted.size());
+  if (st == HMG_OK) st = upload(&db->d_order, db->order.data(), db->order.size());
+  if (st == HMG_OK) st = upload(&db->d_inv, inv.data(), inv.size());
+  if (st == HMG_OK) st = upload(&db->d_tjb, tjb.data(), tjb.size());
+  if (st == HMG_OK) st = upload(&db->d_move, mv.data(), mv.size());
+  if (st != HMG_OK) {
+    hmg_db_destroy(db);
+    return st;
+  }
+  *out = db;
+  return HMG_OK;
+}
+
+int64_t hmg_db_nseq(const hmg_db* db) { return db ? db->nseq : -1; }
+int64_t hmg_db_residues(const hmg_db* db) { return db ? db->residues : -1; }
+int64_t hmg_db_packed_bytes(const hmg_db* db) { return db ? std::max<int64_t>(db->nwords, 4) * 4 : -1; }
+
+hmg_status hmg_db_order(const hmg_db* db, int32_t* order) {
+  if (!db || (!order && db->nseq)) return HMG_EINVAL;
+  std::copy(db->order.begin(), db->order.end(), order);
+  return HMG_OK;
+}
+
+hmg_status hmg_db_image(const hmg_db* db, uint32_t* image) {
+  if (!db || !image) return HMG_EINVAL;
+  if (db->device < 0) {
+    std::copy(db->host_image.begin(), db->host_image.end(), image);
+    return HMG_OK;
+  }
+  Dev dg(db->device);
+  return cuda_status(cudaMemcpy(image, db->d_words, (size_t)hmg_db_packed_bytes(db), cudaMemcpyDeviceToHost));
+}
+
+hmg_status hmg_db_upload(hmg_db* db, const uint32_t* image, void* stream) {
+  if (!db || !image || db->device < 0) return HMG_EINVAL;
+  Dev dg(db->device);
+  return cuda_status(cudaMemcpyAsync(db->d_words, image, (size_t)hmg_db_packed_bytes(db), cudaMemcpyHostToDevice,
+                                     (cudaStream_t)stream));
+}
+
+void hmg_db_destroy(hmg_db* db) {
+  if (!db) return;
+  if (db->device >= 0) {
+    Dev dg(db->device);
+    cudaFree(db->d_words);
+    cudaFree(db->d_woff16);
+    cudaFree(db->d_len);
+    cudaFree(db->d_order);
+    cudaFree(db->d_inv);
+    cudaFree(db->d_tjb);
+    cudaFree(db->d_move);
+    cudaGetLastError();
+  }
+  delete db;
+}
+
+hmg_status hmg_msv(const hmg_profile* pc, const hmg_db* db, double F1, void* stream, uint8_t* raw, uint8_t* pass) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !db || (!raw && db->nseq) || p->device != db->device || db->device < 0) return HMG_EINVAL;
+  if (pass && (!p->has_ev || !(F1 > 0.0 && F1 <= 1.0))) return HMG_EINVAL;
+  if (db->nseq == 0) return HMG_OK;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint16_t* thr = nullptr;
+  if (pass) {
+    hmg_status s = msv_thr_table(p, db, F1, &thr);
+    if (s != HMG_OK) return s;
+  }
+  cudaError_t e = cudaSuccess;
+  hmg_status s;
+  {
+    Scratch S(st);
+    auto* raw_sorted = (uint8_t*)S.get((size_t)db->nseq, &e);
+    void* tmp = S.get(scan_tmp_bytes(db->nseq) + (size_t)db->nseq + 16, &e);
+    if (e) return cuda_status(e);
+    mark_reset();
+    s = run_msv(p, db, st, raw_sorted, S);
+    if (s != HMG_OK) return s;
+    e = msv_finish(raw_sorted, db->d_len, db->d_order, db->nseq, thr, raw, pass, nullptr, nullptr, nullptr, tmp,
+                   st);
+    mark(3, st);
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  return cuda_status(e);
+}
+
+hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* ids, int64_t n, double F2,
+                       void* stream, int16_t* raw, uint8_t* pass) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !db || !p->has_tsc || (!raw && db->nseq) || p->device != db->device || db->device < 0)
+    return HMG_EINVAL;
+  if (pass && (!p->has_ev || !(F2 > 0.0 && F2 <= 1.0))) return HMG_EINVAL;
+  if (ids && n < 0) return HMG_EINVAL;
+  if (db->nseq == 0 || (ids && n == 0)) return HMG_OK;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const int32_t* thr = nullptr;
+  if (pass) {
+    hmg_status s = vit_thr_table(p, db, F2, &thr);
+    if (s != HMG_OK) return s;
+  }
+  cudaError_t e = cudaSuccess;
+  {
+    Scratch S(st);
+    auto* raw_sorted = (int16_t*)S.get(sizeof(int16_t) * (size_t)db->nseq, &e);
+    if (e) return cuda_status(e);
+    const int32_t* list = nullptr;
+    const int64_t* nl = nullptr;
+    int64_t nmax = db->nseq;
+    if (ids) {
+      auto* sl = (int32_t*)S.get(sizeof(int32_t) * (size_t)n, &e);
+      auto* cnt = (int64_t*)S.get(sizeof(int64_t), &e);
+      if (e) return cuda_status(e);
+      if ((e = to_sorted_ids(ids, n, db->d_inv, sl, st))) return cuda_status(e);
+      if ((e = set_count(cnt, n, st))) return cuda_status(e);
+      list = sl;
+      nl = cnt;
+      nmax = n;
+    }
+    mark_reset();
+    hmg_status s = run_vit(p, db, list, nl, st, raw_sorted, S);
+    if (s != HMG_OK) return s;
+    e = vit_finish(raw_sorted, list, nl, nmax, db->d_len, db->d_order, thr, raw, pass, nullptr, st);
+    mark(5, st);
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  return cuda_status(e);
+}
+
+hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
+                        uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                        int64_t* n_survivors) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !db || !p->has_tsc || !p->has_ev || p->device != db->device || db->device < 0) return HMG_EINVAL;
+  if (!(F1 > 0.0 && F1 <= 1.0) || !(F2 > 0.0 && F2 <= 1.0)) return HMG_EINVAL;
+  if (db->nseq && (!msv_raw || !vit_raw || !flags || !survivor_ids || !n_survivors)) return HMG_EINVAL;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  if (db->nseq == 0) return n_survivors ? cuda_status(set_count(n_survivors, 0, st)) : HMG_OK;
+  const uint16_t* tm = nullptr;
+  const int32_t* tv = nullptr;
+  hmg_status s = msv_thr_table(p, db, F1, &tm);
+  if (s == HMG_OK) s = vit_thr_table(p, db, F2, &tv);
+  if (s != HMG_OK) return s;
+  cudaError_t e = cudaSuccess;
+  {
+    Scratch S(st);
+    const int64_t n = db->nseq;
+    auto* raw_sorted = (uint8_t*)S.get((size_t)n, &e);
+    auto* vraw_sorted = (int16_t*)S.get(sizeof(int16_t) * (size_t)n, &e);
+    auto* surv = (int32_t*)S.get(sizeof(int32_t) * (size_t)n, &e);
+    void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
+    if (e) return cuda_status(e);
+    mark_reset();
+    s = run_msv(p, db, st, raw_sorted, S);                                   // Fig 1: MSV
+    if (s != HMG_OK) return s;
+    e = msv_finish(raw_sorted, db->d_len, db->d_order, n, tm, msv_raw, flags, surv, n_survivors, survivor_ids, tmp,
+                   st);                                                       // pass + compaction
+    if (e) return cuda_status(e);
+    s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S);               // P7Viterbi on survivors
+    if (s != HMG_OK) return s;
+    e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st);
+    mark(5, st);
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  return cuda_status(e);
+}
+
+}  // extern "C"

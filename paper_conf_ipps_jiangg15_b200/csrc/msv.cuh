@@ -1,0 +1,175 @@
+// msv.cuh -- MSV filter kernels for sm_100a (Alg 1).
+//
+// Fast kernel (msv_fast_kernel<G, Q>): a group of G lanes scores one sequence
+// (the paper's "warp = one sequence", generalised to G in
+// {4, 8, 16, 32}); 32/G sequences of equal length rank share a warp.  Each lane
+// holds Q 32-bit registers of DP cells as s16x2 pairs (HMMER's Farrar striping,
+// ref [19], over 2G virtual lanes: register q of lane z holds nodes z*Q+q+1 (low
+// half) and (z+G)*Q+q+1 (high half)), so the diagonal dependence of Alg 1 l.15
+// is register q-1 -> q inside a lane and one __shfl_sync per row across lanes
+// (the paper's double buffering, becomes register renaming).
+//
+// Cell update: the state of a cell is
+//     t_i[k] = max(s_{i-1}[k-1] + bias, B')        with B' = min(xB - tbm + bias, 255)
+// and one row is a single DPX instruction per register,
+//     t_{i+1}[k+1] = VIADDMNMX.S16x2(t_i[k], e[x_i][k], B')    e = bias - cost,
+// which reproduces Alg 1 l.15 (max, +bias, -cost, all u8-saturating) exactly
+// while no row has overflowed (proof in DESIGN.md; the u8 floor at 0 is
+// absorbed by B' >= bias).  xE (Alg 1 l.16/l.20) is tracked as a running
+// per-lane max R (VIMNMX3, half an instruction per register) and a per-row
+// __ballot_sync against the threshold at which J->B or overflow could change;
+// B' is speculated unchanged and corrected (monotone max) on the rare rows
+// where the vote fires.  Valid iff bias < 66 + tbm (host check); otherwise the
+// exact kernel runs.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "hmg_internal.h"
+
+namespace hmg {
+
+// The striped table row layout for (G, Q): chunks of 4, then 2, then 1 words per
+// lane; chunk c occupies G*w_c consecutive words, lane z at offset z*w_c.
+template <int Q>
+struct Chunks {
+  static constexpr int n4 = Q / 4;
+  static constexpr int r = Q % 4;
+  static constexpr bool has2 = r >= 2;
+  static constexpr bool has1 = (r % 2) == 1;
+};
+
+template <int G, int Q>
+__device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z, uint32_t (&e)[Q]) {
+  using C = Chunks<Q>;
+#pragma unroll
+  for (int c = 0; c < C::n4; ++c) {
+    uint4 v = *reinterpret_cast<const uint4*>(row + c * 4 * G + z * 4);
+    e[4 * c + 0] = v.x;
+    e[4 * c + 1] = v.y;
+    e[4 * c + 2] = v.z;
+    e[4 * c + 3] = v.w;
+  }
+  if constexpr (C::has2) {
+    uint2 v = *reinterpret_cast<const uint2*>(row + C::n4 * 4 * G + z * 2);
+    e[4 * C::n4 + 0] = v.x;
+    e[4 * C::n4 + 1] = v.y;
+  }
+  if constexpr (C::has1) {
+    e[Q - 1] = row[(C::n4 * 4 + (C::has2 ? 2 : 0)) * G + z];
+  }
+}
+
+__device__ __forceinline__ int msv_thr(int xJ, int bias) {
+  // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
+  int T = max(xJ, 189) + 4;
+  T = min(T, 255 - bias);
+  return T + bias;
+}
+
+template <int G, int Q>
+__global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
+  extern __shared__ uint4 smem4[];
+  uint32_t* sm = reinterpret_cast<uint32_t*>(smem4);
+  constexpr int ROWW = Q * G;              // words per residue row
+  constexpr int NG = 32 / G;               // sequences per warp
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(a.prof);
+    for (int i = threadIdx.x; i < kRows * ROWW / 4; i += blockDim.x) smem4[i] = src[i];
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const int z = lane & (G - 1);
+  const int grp = lane / G;
+  const unsigned gbits = (G == 32 ? 0xffffffffu : ((1u << G) - 1u)) << (grp * G);
+  const uint32_t sel = (z == 0) ? 0x1054u : 0x3210u;   // carry fix-up for virtual lane 0 / G
+  const uint32_t negpair = (uint32_t)(uint16_t)kNegE;  // low half = -inf
+  const int bias = a.bias, tbm = a.tbm;
+
+  for (;;) {
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(a.counter, (unsigned long long)NG);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if ((long long)base >= a.nseq) break;
+    const long long s = (long long)base + grp;
+    const bool valid = s < a.nseq;
+    const int L = valid ? a.len[s] : 0;
+    const int Lmax = __shfl_sync(0xffffffffu, L, 0);   // sorted by length, descending
+    const uint32_t* wp = a.words + (valid ? (size_t)a.woff16[s] * 4 : 0);
+    const int nw = (L + 5) / 6;
+    const int tjb = valid ? a.tjb[L] : 0;
+
+    int xJ = 0;
+    bool ovf = false;
+    int Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
+    uint32_t B2 = (uint32_t)Bp * 0x10001u;
+    uint32_t thrv = (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u;
+    if (!valid) thrv = 0;   // never fires
+
+    uint32_t t[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
+    uint32_t R = B2;
+
+    const int nblk = (Lmax + 5) / 6;
+    uint32_t wnext = (0 < nw) ? __ldg(wp) : 0xffffffffu;
+    for (int blk = 0; blk < nblk; ++blk) {
+      const uint32_t w = wnext;
+      wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
+#pragma unroll
+      for (int j = 0; j < 6; ++j) {
+        const int x = (w >> (5 * j)) & 31;
+        uint32_t e[Q];
+        load_row<G, Q>(sm + x * ROWW, z, e);
+        // diagonal carry from the previous virtual lane (value after its emission)
+        uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
+        c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
+        c = __byte_perm(c, negpair, sel);
+#pragma unroll
+        for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
+        t[0] = __vmaxs2(c, B2);
+#pragma unroll
+        for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
+        if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+        // does any cell of this row reach the J->B / overflow threshold?
+        const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
+        const unsigned bal = __ballot_sync(0xffffffffu, hit);
+        if (bal) {
+          uint32_t m = R;
+#pragma unroll
+          for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
+          const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
+          if ((bal & gbits) && !ovf) {
+            if (Rmax >= 255) {           // xE >= 255 - bias: overflow (reading R13)
+              ovf = true;
+              thrv = 0;
+            } else {
+              xJ = max(xJ, Rmax - bias - 3);                 // E->J, Alg 1 l.20
+              const int xB = max(kBaseB, xJ) - tjb;          // J->B
+              Bp = min(max(xB - tbm, 0) + bias, 255);
+              B2 = (uint32_t)Bp * 0x10001u;
+#pragma unroll
+              for (int q = 0; q < Q; ++q) t[q] = __vmaxs2(t[q], B2);
+              thrv = (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u;
+            }
+          }
+        }
+      }
+    }
+    // final xJ = max over all cells of (s - 3); R holds max over t = max(s + bias, B')
+    uint32_t m = R;
+#pragma unroll
+    for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
+    if (valid && z == 0) {
+      int raw;
+      if (ovf) raw = 255;
+      else if (Rmax > Bp) raw = max(xJ, max(Rmax - bias - 3, 0));
+      else raw = 254;                 // every cell <= B': exact kernel recomputes (rare)
+      a.raw[s] = (uint8_t)raw;
+    }
+  }
+}
+
+}  // namespace hmg

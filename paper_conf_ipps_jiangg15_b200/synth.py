@@ -123,18 +123,14 @@ _CDF = np.concatenate([np.cumsum(BACKGROUND * (1.0 - _PX)), [1.0]])
 _SYMS = np.concatenate([np.arange(NCANON), [CODE_X]]).astype(np.uint8)
 
 
-def _residues(key: int, start: int, n: int) -> np.ndarray:
-    """Residues at global positions [start, start+n) of DB stream ``key``."""
-    out = np.empty(n, dtype=np.uint8)
-    step = 1 << 22
+# 16-bit inverse-CDF table: a residue is _TABLE[top 16 bits of splitmix64(position ^ key)]
+_TABLE = _SYMS[np.searchsorted(_CDF, (np.arange(65536) + 0.5) / 65536.0, side="right").clip(0, NCANON)]
+
+
+def _residues_at(key: int, pos: np.ndarray) -> np.ndarray:
+    """Residues at global positions ``pos`` (uint64) of DB stream ``key``."""
     k = np.uint64((int(key) * 0xD1B54A32D192ED03) & 0xFFFFFFFFFFFFFFFF)
-    for a in range(0, n, step):
-        b = min(n, a + step)
-        pos = np.arange(start + a, start + b, dtype=np.uint64)
-        with np.errstate(over="ignore"):
-            u = (_splitmix64(pos ^ k) >> np.uint64(11)).astype(np.float64) * (1.0 / 9007199254740992.0)
-        out[a:b] = _SYMS[np.searchsorted(_CDF, u, side="right").clip(0, NCANON)]
-    return out
+    return _TABLE[(_splitmix64(pos ^ k) >> np.uint64(48)).astype(np.intp)]
 
 
 class Database:
@@ -160,16 +156,18 @@ class Database:
         L = self.lengths[ids].astype(np.int64)
         off = np.zeros(len(ids) + 1, dtype=np.int64)
         np.cumsum(L, out=off[1:])
-        dsq = np.empty(int(off[-1]), dtype=np.uint8)
-        # contiguous runs of ids map to contiguous global positions: batch them
-        if len(ids):
-            brk = np.nonzero(np.diff(ids) != 1)[0] + 1
-            starts = np.concatenate([[0], brk])
-            ends = np.concatenate([brk, [len(ids)]])
-            for s, e in zip(starts, ends):
-                g0 = int(self.gstart[ids[s]])
-                g1 = int(self.gstart[ids[e - 1] + 1])
-                dsq[off[s]:off[e]] = _residues(self.seed, g0, g1 - g0)
+        total = int(off[-1])
+        dsq = np.empty(total, dtype=np.uint8)
+        step = 1 << 24
+        shift = self.gstart[ids] - off[:-1]           # global position = local position + shift
+        for a in range(0, total, step):
+            b = min(total, a + step)
+            j0 = int(np.searchsorted(off, a, side="right")) - 1
+            j1 = int(np.searchsorted(off, b - 1, side="right"))
+            lo = np.maximum(off[j0:j1], a)
+            hi = np.minimum(off[j0 + 1:j1 + 1], b)
+            pos = np.repeat(shift[j0:j1], hi - lo) + np.arange(a, b, dtype=np.int64)
+            dsq[a:b] = _residues_at(self.seed, pos.astype(np.uint64))
         if len(self.planted_ids) and self.profile is not None:
             where = {int(s): j for j, s in enumerate(ids)}
             for s in self.planted_ids:

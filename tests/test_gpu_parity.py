@@ -1,0 +1,313 @@
+"""GPU parity: libhmg's CUDA path vs the CPU oracle, bit-exact (raw scores and flags).
+
+Every call goes through the C ABI (paper_conf_ipps_jiangg15_b200.hmg).  Cases
+span several tiles and ragged tails: model lengths around every register /
+lane-group boundary, sequence lengths 1..7 and around the 6-residue word, the
+adversarial profiles (saturating bias, long D->D chains, -inf emissions), and
+the BASELINE configurations (config 1 in full; configs 2/3 at full size on a
+sample the oracle scores one by one).
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ipps_jiangg15_b200 import build, hmg, synth
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test run without a CUDA device")
+    build.build()
+    hmg.lib()
+
+
+def _db_from(dsq_list):
+    off = np.zeros(len(dsq_list) + 1, np.int64)
+    np.cumsum([len(d) for d in dsq_list], out=off[1:])
+    dsq = np.concatenate(dsq_list).astype(np.uint8) if dsq_list else np.zeros(0, np.uint8)
+    return dsq, off
+
+
+def _ragged_db(rng, n=70, alphabet=20, lmax=400):
+    lens = list(range(1, 14)) + [17, 18, 19, 23, 24, 25, 35, 36, 37, 95, 96, 97]
+    lens += rng.integers(1, lmax, size=max(0, n - len(lens))).tolist()
+    return _db_from([synth.random_dsq(rng, int(L), alphabet) for L in lens])
+
+
+def _msv_gpu(prof_msc, dsq, off, **kw):
+    p = hmg.Profile(prof_msc, **kw)
+    db = hmg.Database(dsq, off)
+    raw = torch.zeros(db.nseq, dtype=torch.uint8, device="cuda")
+    hmg.hmg_msv(p, db, raw)
+    torch.cuda.synchronize()
+    return raw.cpu().numpy().astype(np.int32), p
+
+
+def _vit_gpu(msc, tsc, dsq, off, ids=None):
+    p = hmg.Profile(msc, tsc)
+    db = hmg.Database(dsq, off)
+    raw = torch.full((db.nseq,), -12345, dtype=torch.int16, device="cuda")
+    t_ids = None if ids is None else torch.as_tensor(ids, dtype=torch.int32, device="cuda")
+    hmg.hmg_viterbi(p, db, raw, ids=t_ids)
+    torch.cuda.synchronize()
+    return raw.cpu().numpy().astype(np.int32), p
+
+
+# ------------------------------------------------------------------ MSV
+def test_msv_config1_full():
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    got, _ = _msv_gpu(prof.msc, dsq, off)
+    want = oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off)
+    assert np.array_equal(got, want)
+
+
+MS = [1, 2, 3, 4, 5, 7, 8, 9, 15, 16, 17, 31, 32, 33, 48, 63, 64, 65, 100, 127, 128, 129, 200, 255, 256, 257,
+      400, 511, 512, 513, 700, 1000, 1024, 1025, 1528, 2048, 2049, 2405, 2560, 2561, 3000]
+
+
+@pytest.mark.parametrize("M", MS)
+def test_msv_model_lengths(M):
+    rng = np.random.default_rng(M)
+    prof = synth.make_profile(M, 7000 + M)
+    dsq, off = _ragged_db(rng, n=60, alphabet=29)
+    got, _ = _msv_gpu(prof.msc, dsq, off)
+    want = oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off)
+    assert np.array_equal(got, want)
+
+
+@pytest.mark.parametrize("G", [4, 8, 16, 32])
+@pytest.mark.parametrize("M", [60, 333, 900])
+def test_msv_every_lane_group(G, M, monkeypatch):
+    monkeypatch.setenv("HMG_MSV_G", str(G))
+    rng = np.random.default_rng(G * 1000 + M)
+    prof = synth.make_profile(M, M + G, stress=True)
+    dsq, off = _ragged_db(rng, n=90, alphabet=29)
+    got, p = _msv_gpu(prof.msc, dsq, off)
+    q = p.quant()
+    assert q["msv_lanes"] >= G or q["msv_regs"] == 0
+    assert np.array_equal(got, oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off))
+
+
+@pytest.mark.parametrize("score,fast", [(20.0, 1), (22.5, 1), (23.0, 1), (30.0, 0), (45.0, 0)])
+def test_msv_overflow_and_exact_kernel(score, fast):
+    """msc = +20 nats: bias 87 < 66 + tbm -> fast kernel, cells saturate -> raw 255 (R13);
+    msc >= +30 nats: bias >= 66 + tbm -> the exact kernel (fast-kernel precondition)."""
+    rng = np.random.default_rng(1)
+    msc = np.full((40, 29), score, np.float32)
+    msc[:, 25:] = -np.inf
+    msc[::3, 4] = -3.0
+    dsq, off = _ragged_db(rng, n=30, alphabet=29)
+    got, p = _msv_gpu(msc, dsq, off)
+    assert p.quant()["msv_fast"] == fast
+    assert np.array_equal(got, oracle.msv_db(oracle.MSVProfile(msc), dsq, off))
+    assert (got == 255).sum() > 0
+
+
+def test_msv_high_scores_fast_path():
+    """Strong hits: planted homologs and a high-scoring profile drive the J->B update
+    (vote fires) and the in-kernel overflow test of the fast kernel."""
+    rng = np.random.default_rng(3)
+    prof = synth.make_profile(150, 99)
+    msc = prof.msc.copy()
+    msc[:, :20] *= 1.9          # higher bias, still fast
+    p_or = oracle.MSVProfile(msc)
+    seqs = []
+    for i in range(80):
+        L = int(rng.integers(20, 600))
+        d = synth.random_dsq(rng, L)
+        seg = np.argmax(msc[:, :20], axis=1)[: min(L, 150 - (i % 40))].astype(np.uint8)
+        a = int(rng.integers(0, L - len(seg) + 1))
+        if i % 3:
+            d[a:a + len(seg)] = seg
+        seqs.append(d)
+    dsq, off = _db_from(seqs)
+    got, p = _msv_gpu(msc, dsq, off)
+    assert p.quant()["msv_fast"] == 1
+    want = oracle.msv_db(p_or, dsq, off)
+    assert np.array_equal(got, want)
+    assert (want == 255).sum() > 0 and (want >= 190).sum() > 0
+
+
+def test_msv_all_minus_inf_redo_path():
+    """Gap-only sequences: every cell <= B', the fast kernel defers to the exact kernel."""
+    prof = synth.make_profile(77, 5)
+    seqs = [np.full(L, 20, np.uint8) for L in (1, 2, 6, 7, 50)] + [np.array([27, 28, 20], np.uint8)]
+    dsq, off = _db_from(seqs)
+    got, _ = _msv_gpu(prof.msc, dsq, off)
+    assert np.array_equal(got, oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off))
+
+
+def test_empty_db():
+    prof = synth.make_profile(10, 1)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=(-9, math.log(2), -9, math.log(2)))
+    db = hmg.Database(np.zeros(0, np.uint8), np.zeros(1, np.int64))
+    out = hmg.alloc_outputs(0)
+    hmg.hmg_pipeline(p, db, **out)
+    torch.cuda.synchronize()
+    assert int(out["n_survivors"].item()) == 0
+
+
+# ------------------------------------------------------------------ Viterbi
+def test_vit_config1_full():
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    got, _ = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+    want = oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)
+    assert np.array_equal(got, want)
+
+
+VMS = [1, 2, 3, 4, 5, 8, 9, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 200, 255, 256, 257, 400, 511,
+       512, 513, 1000, 2048]
+
+
+@pytest.mark.parametrize("M", VMS)
+@pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
+def test_vit_model_lengths(M, dd):
+    rng = np.random.default_rng(M + int(dd[0]))
+    prof = synth.make_profile(M, 8000 + M, dd=dd)
+    n = 40 if M <= 600 else 12
+    dsq, off = _ragged_db(rng, n=n, alphabet=29, lmax=300)
+    got, _ = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off))
+
+
+@pytest.mark.parametrize("M", [3, 20, 64, 130, 300, 500, 700])
+def test_vit_long_delete_chains(M):
+    """Entry only at node 1, good matches only at nodes 1 and M: the score depends on
+    D->D chains that cross every lane boundary (Lazy-F carries, Fig 7)."""
+    rng = np.random.default_rng(M)
+    msc = np.full((M, 29), -6.0, np.float32)
+    msc[0, 0] = 4.0
+    msc[M - 1, 1] = 4.0
+    tsc = np.log(rng.uniform(0.05, 1.0, size=(M, 8))).astype(np.float32)
+    tsc[:, 7] = np.log(rng.uniform(0.8, 0.999, size=M))
+    tsc[1:, 0] = -np.inf
+    tsc[0, 1:4] = -np.inf
+    tsc[M - 1, 4:8] = -np.inf
+    seqs = [np.array([0, 1], np.uint8), np.array([0, 2, 1], np.uint8), np.array([0, 1, 0, 1], np.uint8)]
+    seqs += [synth.random_dsq(rng, int(L), 3) for L in rng.integers(1, 60, size=30)]
+    dsq, off = _db_from(seqs)
+    got, _ = _vit_gpu(msc, tsc, dsq, off)
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
+
+
+def test_vit_overflow_and_minus_inf():
+    rng = np.random.default_rng(4)
+    M = 50
+    msc = np.full((M, 29), 60.0, np.float32)
+    msc[:, 10:] = -np.inf
+    tsc = np.full((M, 8), np.log(0.3), np.float32)
+    tsc[0, 1:4] = -np.inf
+    tsc[-1, 4:] = -np.inf
+    dsq, off = _ragged_db(rng, n=30, alphabet=29, lmax=100)
+    got, _ = _vit_gpu(msc, tsc, dsq, off)
+    want = oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off)
+    assert np.array_equal(got, want)
+    assert (want == 32767).any() and (want < 0).any()
+
+
+def test_vit_ids_subset_untouched_elsewhere():
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    ids = np.array([5, 3, 3, 999, 0, 512], np.int32)
+    got, _ = _vit_gpu(prof.msc, prof.tsc, dsq, off, ids=ids)
+    want = oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off, ids=ids)
+    assert np.array_equal(got[ids], want)
+    mask = np.ones(len(got), bool)
+    mask[ids] = False
+    assert (got[mask] == -12345).all()
+
+
+# ------------------------------------------------------------------ pipeline + flags
+def _calibrate(prof):
+    """mu for lambda = ln 2 fitted by the ORACLE on 1000 background sequences of L = 200."""
+    cal = synth.Database(np.full(1000, 200, np.int32), seed=7)
+    dsq, off = cal.materialize()
+    mp, vp = oracle.MSVProfile(prof.msc), oracle.VitProfile(prof.msc, prof.tsc)
+    lam = math.log(2)
+    mb = [oracle.bits(oracle.msv_nats(int(r), 200), 200) for r in oracle.msv_db(mp, dsq, off)]
+    vb = [oracle.bits(oracle.vit_nats(int(r), 200), 200) for r in oracle.vit_db(vp, dsq, off)]
+    return (oracle.fit_mu(np.array(mb), lam), lam, oracle.fit_mu(np.array(vb), lam), lam)
+
+
+def _check_pipeline(prof, dsq, off, F1, F2, sample=None):
+    ev = _calibrate(prof)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    db = hmg.Database(dsq, off)
+    out = hmg.alloc_outputs(db.nseq)
+    hmg.hmg_pipeline(p, db, F1=F1, F2=F2, **out)
+    torch.cuda.synchronize()
+    mraw = out["msv_raw"].cpu().numpy().astype(np.int32)
+    vraw = out["vit_raw"].cpu().numpy().astype(np.int32)
+    flags = out["flags"].cpu().numpy()
+    ns = int(out["n_survivors"].item())
+    surv = out["survivor_ids"].cpu().numpy()[:ns]
+    lens = np.diff(off)
+    mp, vp = oracle.MSVProfile(prof.msc), oracle.VitProfile(prof.msc, prof.tsc)
+    idx = np.arange(db.nseq) if sample is None else np.asarray(sample)
+    want_m = oracle.msv_db(mp, dsq, off, ids=idx)
+    assert np.array_equal(mraw[idx], want_m)
+    want_pass = np.array([oracle.msv_pass(int(r), int(lens[s]), ev[0], ev[1], F1) for r, s in zip(want_m, idx)])
+    assert np.array_equal(flags[idx] & 1, want_pass)
+    # survivors: exactly the MSV-passing sequences, length-descending, stable (caller order on ties)
+    passing = np.nonzero(flags & 1)[0]
+    assert sorted(surv.tolist()) == passing.tolist()
+    order = np.lexsort((np.arange(db.nseq), -lens))
+    assert surv.tolist() == [s for s in order if flags[s] & 1]
+    # Viterbi ran on every survivor and only there
+    assert np.array_equal((flags >> 2) & 1, flags & 1)
+    assert (vraw[flags & 1 == 0] == -32768).all()
+    vs = surv if sample is None else np.intersect1d(surv, idx)
+    want_v = oracle.vit_db(vp, dsq, off, ids=vs)
+    assert np.array_equal(vraw[vs], want_v)
+    want_vp = np.array([oracle.vit_pass(int(r), int(lens[s]), ev[2], ev[3], F2) for r, s in zip(want_v, vs)])
+    assert np.array_equal((flags[vs] >> 1) & 1, want_vp.astype(np.uint8))
+    return ns
+
+
+def test_pipeline_config1():
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    ns = _check_pipeline(prof, dsq, off, F1=0.02, F2=1e-3)
+    assert 0 < ns < 200
+
+
+def test_pipeline_loose_thresholds():
+    """F1 = 0.5 sends about half the DB to the Viterbi stage; F = 1 passes everything."""
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    ns = _check_pipeline(prof, dsq, off, F1=0.5, F2=0.5)
+    assert ns > 300
+    assert _check_pipeline(prof, dsq, off, F1=1.0, F2=1.0) == db.N
+
+
+def test_pipeline_config3_full_size_sampled():
+    """BASELINE config 3 at full size (550k sequences, M=400, planted homologs) in the
+    bench launch configuration; the oracle checks a length-stratified sample plus
+    every survivor in it."""
+    prof, db = synth.config(3)
+    dsq, off = db.materialize()
+    rng = np.random.default_rng(0)
+    sample = np.unique(np.concatenate([rng.choice(db.N, 3000, replace=False), db.planted_ids,
+                                       np.argsort(-db.lengths)[:50]]))
+    _check_pipeline(prof, dsq, off, F1=0.02, F2=1e-3, sample=sample)
+
+
+def test_msv_config2_full_size_sampled():
+    prof, db = synth.config(2)
+    dsq, off = db.materialize()
+    got, _ = _msv_gpu(prof.msc, dsq, off)
+    rng = np.random.default_rng(1)
+    sample = np.unique(np.concatenate([rng.choice(db.N, 4000, replace=False), np.argsort(-db.lengths)[:40],
+                                       np.argsort(db.lengths)[:40]]))
+    want = oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off, ids=sample)
+    assert np.array_equal(got[sample], want)
