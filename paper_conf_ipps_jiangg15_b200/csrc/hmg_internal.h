@@ -26,6 +26,7 @@ struct MsvArgs {
   const uint32_t* woff16;    // [nseq] sorted: word offset / 4 (16-byte units)
   const int32_t* len;        // [nseq] sorted lengths (descending)
   int64_t nseq;
+  int64_t nlong;             // fast kernel: the first nlong sorted sequences go to the G=32 queue
   const uint8_t* tjb;        // [Lmax+1] tjb_b(L)
   const uint32_t* prof;      // striped s16x2 emission table for (G, Q), kRows rows
   const uint8_t* cost;       // plain biased costs [kRows][M] (exact kernel)

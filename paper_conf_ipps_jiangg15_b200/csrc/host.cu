@@ -347,6 +347,14 @@ hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
   a.raw = raw_sorted;
+  // long sequences: L > max(1000, 8 x mean length) (env HMG_MSV_LLONG overrides), length-sorted prefix
+  {
+    const double mean = n ? (double)db->residues / (double)n : 0.0;
+    const int llong = env_int("HMG_MSV_LLONG", (int)std::max(1000.0, 8.0 * mean));
+    const auto it = std::upper_bound(db->len_sorted.begin(), db->len_sorted.end(), llong,
+                                     [](int v, int L) { return v > L; });
+    a.nlong = (int64_t)(it - db->len_sorted.begin());
+  }
   auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
@@ -562,6 +570,11 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   }
   if (st == HMG_OK && p->msv_Q > 0) {
     auto t = msv_table(*p, p->msv_G, p->msv_Q);
+    if (p->msv_G < 32) {   // second table for the whole-warp (G = 32) long-sequence queue
+      const int QL = (p->msv_G * p->msv_Q + 31) / 32;
+      auto t2 = msv_table(*p, 32, QL);
+      t.insert(t.end(), t2.begin(), t2.end());
+    }
     p->msv_prof_bytes = t.size() * 4;
     st = upload(&p->d_msv_prof, t.data(), t.size());
   }

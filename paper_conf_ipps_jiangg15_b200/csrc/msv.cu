@@ -34,7 +34,8 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
   const void* fn = msv_fast_ptr(G, Q);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
-  const size_t smem = (size_t)kRows * Q * G * 4;
+  const int QL = (G == 32) ? 0 : (G * Q + 31) / 32;
+  const size_t smem = ((size_t)kRows * Q * G + (size_t)kRows * QL * 32) * 4;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = 0, per = 0;

@@ -67,18 +67,12 @@ __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   return T + bias;
 }
 
+// Score one batch of 32/G sequences (sorted indices s0 + group) with G lanes per
+// sequence and Q s16x2 registers per lane, profile table `sm` in shared memory.
 template <int G, int Q>
-__global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
-  extern __shared__ uint4 smem4[];
-  uint32_t* sm = reinterpret_cast<uint32_t*>(smem4);
+__device__ __forceinline__ void msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
+                                          long long send) {
   constexpr int ROWW = Q * G;              // words per residue row
-  constexpr int NG = 32 / G;               // sequences per warp
-  {
-    const uint4* src = reinterpret_cast<const uint4*>(a.prof);
-    for (int i = threadIdx.x; i < kRows * ROWW / 4; i += blockDim.x) smem4[i] = src[i];
-  }
-  __syncthreads();
-
   const int lane = threadIdx.x & 31;
   const int z = lane & (G - 1);
   const int grp = lane / G;
@@ -87,88 +81,123 @@ __global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
   const uint32_t negpair = (uint32_t)(uint16_t)kNegE;  // low half = -inf
   const int bias = a.bias, tbm = a.tbm;
 
-  for (;;) {
-    unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(a.counter, (unsigned long long)NG);
-    base = __shfl_sync(0xffffffffu, base, 0);
-    if ((long long)base >= a.nseq) break;
-    const long long s = (long long)base + grp;
-    const bool valid = s < a.nseq;
-    const int L = valid ? a.len[s] : 0;
-    const int Lmax = __shfl_sync(0xffffffffu, L, 0);   // sorted by length, descending
-    const uint32_t* wp = a.words + (valid ? (size_t)a.woff16[s] * 4 : 0);
-    const int nw = (L + 5) / 6;
-    const int tjb = valid ? a.tjb[L] : 0;
+  const long long s = s0 + grp;
+  const bool valid = s < send;
+  const int L = valid ? a.len[s] : 0;
+  int Lmax = L;                                         // sorted descending: group 0 is the longest
+  if constexpr (G < 32) Lmax = __shfl_sync(0xffffffffu, L, 0);
+  const uint32_t* wp = a.words + (valid ? (size_t)a.woff16[s] * 4 : 0);
+  const int nw = (L + 5) / 6;
+  const int tjb = valid ? a.tjb[L] : 0;
 
-    int xJ = 0;
-    bool ovf = false;
-    int Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
-    uint32_t B2 = (uint32_t)Bp * 0x10001u;
-    uint32_t thrv = (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u;
-    if (!valid) thrv = 0;   // never fires
+  int xJ = 0;
+  bool ovf = false;
+  int Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
+  uint32_t B2 = (uint32_t)Bp * 0x10001u;
+  uint32_t thrv = valid ? (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u : 0u;   // 0: never fires
 
-    uint32_t t[Q];
+  uint32_t t[Q];
 #pragma unroll
-    for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
-    uint32_t R = B2;
+  for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
+  uint32_t R = B2;
 
-    const int nblk = (Lmax + 5) / 6;
-    uint32_t wnext = (0 < nw) ? __ldg(wp) : 0xffffffffu;
-    for (int blk = 0; blk < nblk; ++blk) {
-      const uint32_t w = wnext;
-      wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
+  const int nblk = (Lmax + 5) / 6;
+  uint32_t wnext = (0 < nw) ? __ldg(wp) : 0xffffffffu;
+  for (int blk = 0; blk < nblk; ++blk) {
+    const uint32_t w = wnext;
+    wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
 #pragma unroll
-      for (int j = 0; j < 6; ++j) {
-        const int x = (w >> (5 * j)) & 31;
-        uint32_t e[Q];
-        load_row<G, Q>(sm + x * ROWW, z, e);
-        // diagonal carry from the previous virtual lane (value after its emission)
-        uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
-        c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
-        c = __byte_perm(c, negpair, sel);
+    for (int j = 0; j < 6; ++j) {
+      const int x = (w >> (5 * j)) & 31;
+      uint32_t e[Q];
+      load_row<G, Q>(sm + x * ROWW, z, e);
+      // diagonal carry from the previous virtual lane (value after its emission)
+      uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
+      c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
+      c = __byte_perm(c, negpair, sel);
 #pragma unroll
-        for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
-        t[0] = __vmaxs2(c, B2);
+      for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
+      t[0] = __vmaxs2(c, B2);
 #pragma unroll
-        for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
-        if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
-        // does any cell of this row reach the J->B / overflow threshold?
-        const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
-        const unsigned bal = __ballot_sync(0xffffffffu, hit);
-        if (bal) {
-          uint32_t m = R;
+      for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
+      if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+      // does any cell of this row reach the J->B / overflow threshold?
+      const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
+      const unsigned bal = __ballot_sync(0xffffffffu, hit);
+      if (bal) {
+        uint32_t m = R;
 #pragma unroll
-          for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
-          const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
-          if ((bal & gbits) && !ovf) {
-            if (Rmax >= 255) {           // xE >= 255 - bias: overflow (reading R13)
-              ovf = true;
-              thrv = 0;
-            } else {
-              xJ = max(xJ, Rmax - bias - 3);                 // E->J, Alg 1 l.20
-              const int xB = max(kBaseB, xJ) - tjb;          // J->B
-              Bp = min(max(xB - tbm, 0) + bias, 255);
-              B2 = (uint32_t)Bp * 0x10001u;
+        for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
+        const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
+        if ((bal & gbits) && !ovf) {
+          if (Rmax >= 255) {           // xE >= 255 - bias: overflow (reading R13)
+            ovf = true;
+            thrv = 0;
+          } else {
+            xJ = max(xJ, Rmax - bias - 3);                 // E->J, Alg 1 l.20
+            const int xB = max(kBaseB, xJ) - tjb;          // J->B
+            Bp = min(max(xB - tbm, 0) + bias, 255);
+            B2 = (uint32_t)Bp * 0x10001u;
 #pragma unroll
-              for (int q = 0; q < Q; ++q) t[q] = __vmaxs2(t[q], B2);
-              thrv = (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u;
-            }
+            for (int q = 0; q < Q; ++q) t[q] = __vmaxs2(t[q], B2);
+            thrv = (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u;
           }
         }
       }
     }
-    // final xJ = max over all cells of (s - 3); R holds max over t = max(s + bias, B')
-    uint32_t m = R;
+  }
+  // final xJ = max over all cells of (s - 3); R holds max over t = max(s + bias, B')
+  uint32_t m = R;
 #pragma unroll
-    for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
-    const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
-    if (valid && z == 0) {
-      int raw;
-      if (ovf) raw = 255;
-      else if (Rmax > Bp) raw = max(xJ, max(Rmax - bias - 3, 0));
-      else raw = 254;                 // every cell <= B': exact kernel recomputes (rare)
-      a.raw[s] = (uint8_t)raw;
+  for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
+  const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
+  if (valid && z == 0) {
+    int raw;
+    if (ovf) raw = 255;
+    else if (Rmax > Bp) raw = max(xJ, max(Rmax - bias - 3, 0));
+    else raw = 254;                 // every cell <= B': exact kernel recomputes (rare)
+    a.raw[s] = (uint8_t)raw;
+  }
+}
+
+// Long sequences (the first a.nlong in length order) use a whole warp (G = 32,
+// QL registers) so their row latency stays well below the kernel's duration;
+// the rest use G lanes.  Two work queues, long first.
+template <int G, int Q>
+struct MsvLong {
+  static constexpr int QL = (G == 32) ? 0 : (G * Q + 31) / 32;
+};
+
+template <int G, int Q>
+__global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
+  extern __shared__ uint4 smem4[];
+  constexpr int QL = MsvLong<G, Q>::QL;
+  constexpr int W0 = kRows * Q * G;        // words of the main table
+  constexpr int W1 = kRows * QL * 32;      // words of the long-sequence table
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(a.prof);
+    for (int i = threadIdx.x; i < (W0 + W1) / 4; i += blockDim.x) smem4[i] = src[i];
+  }
+  __syncthreads();
+  const uint32_t* sm = reinterpret_cast<const uint32_t*>(smem4);
+  const int lane = threadIdx.x & 31;
+  if constexpr (QL > 0) {
+    for (;;) {
+      unsigned long long b = 0;
+      if (lane == 0) b = atomicAdd(a.counter + 1, 1ull);
+      b = __shfl_sync(0xffffffffu, b, 0);
+      if ((long long)b >= a.nlong) break;
+      msv_batch<32, QL>(a, sm + W0, (long long)b, a.nlong);
     }
+  }
+  constexpr int NG = 32 / G;
+  const long long first = (QL > 0) ? a.nlong : 0;
+  for (;;) {
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);
+    b = __shfl_sync(0xffffffffu, b, 0);
+    if (first + (long long)b >= a.nseq) break;
+    msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
   }
 }
 

@@ -70,19 +70,19 @@ def gather(packed, survivor_ids, n_survivors, global_ids, world: int, group=None
     nmax = int(nmax_t.item())
     pad = torch.zeros(nmax, dtype=torch.int32, device=packed.device)
     pad[:n_local] = packed
-    words = torch.empty(world, nmax, dtype=torch.int32, device=packed.device)
+    words = torch.empty(world * nmax, dtype=torch.int32, device=packed.device)
     dist.all_gather_into_tensor(words, pad, group=group)
     gid = torch.full((nmax,), -1, dtype=torch.int64, device=packed.device)
     gid[:n_local] = global_ids
-    gids = torch.empty(world, nmax, dtype=torch.int64, device=packed.device)
+    gids = torch.empty(world * nmax, dtype=torch.int64, device=packed.device)
     dist.all_gather_into_tensor(gids, gid, group=group)
     counts = torch.empty(world, dtype=torch.int64, device=packed.device)
     dist.all_gather_into_tensor(counts, n_survivors.reshape(1), group=group)
     sv = torch.full((nmax,), -1, dtype=torch.int64, device=packed.device)
     sv[:n_local] = global_ids[survivor_ids[:n_local].to(torch.int64).clamp_(0, max(n_local - 1, 0))]
-    surv = torch.empty(world, nmax, dtype=torch.int64, device=packed.device)
+    surv = torch.empty(world * nmax, dtype=torch.int64, device=packed.device)
     dist.all_gather_into_tensor(surv, sv, group=group)
-    return words, gids, counts, surv
+    return words.view(world, nmax), gids.view(world, nmax), counts, surv.view(world, nmax)
 
 
 def assemble(words, gids, counts, surv, n_global: int):

@@ -78,6 +78,7 @@ int main() {
         printf("{\"op\": \"%s\", \"ms\": %.4f, \"Tlaneops_per_s\": %.3f}\n", names[op], ms, instr / ms / 1e9);
     }
   }
+  cudaFuncSetAttribute(lds128, cudaFuncAttributeMaxDynamicSharedMemorySize, 65536);
   for (int rep = 0; rep < 3; ++rep) {
     int iters = 1 << 16;
     cudaEventRecord(e0);
