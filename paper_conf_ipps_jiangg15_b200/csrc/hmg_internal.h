@@ -27,6 +27,7 @@ struct MsvArgs {
   const int32_t* len;        // [nseq] sorted lengths (descending)
   int64_t nseq;
   int64_t nlong;             // fast kernel: the first nlong sorted sequences go to the G=32 queue
+  int skip_long;             // 1: sequences [0, nlong) are scored elsewhere (pipeline long lane)
   const uint8_t* tjb;        // [Lmax+1] tjb_b(L)
   const uint32_t* prof;      // striped s16x2 emission table for (G, Q), kRows rows
   const uint8_t* cost;       // plain biased costs [kRows][M] (exact kernel)
@@ -53,6 +54,18 @@ struct VitArgs {
   int16_t* raw_sorted;       // [nseq] output, sorted order
   unsigned long long* counter;
   int32_t* scratch;          // generic kernel: per-warp rows
+  const uint8_t* done;       // register kernel: skip sorted index s when done[s] (long lane ran it)
+};
+
+// Pipeline long lane: MSV (whole warp) then, on pass, Viterbi (whole warp) for the
+// longest sequences, on SMs it holds exclusively, concurrently with the main MSV kernel.
+struct LongArgs {
+  MsvArgs m;                 // m.prof = whole-warp MSV table (32, QL), m.raw = MSV raw (sorted)
+  VitArgs v;                 // v.rsc / v.tr = register-kernel tables (32, QV), v.raw_sorted
+  const uint16_t* thr;       // MSV pass threshold by length
+  uint8_t* done;             // [nseq] set to 1 where the Viterbi filter ran here
+  int64_t nlong;
+  unsigned long long* counter;
 };
 
 }  // namespace hmg
@@ -75,6 +88,11 @@ struct hmg_profile {
   int16_t* d_rsc = nullptr;         // Viterbi emissions (layout per kernel)
   int32_t* d_tr = nullptr;          // Viterbi transitions (layout per kernel)
   size_t msv_prof_bytes = 0, vit_rsc_bytes = 0, vit_tr_bytes = 0;
+  // pipeline long lane (whole-warp MSV + Viterbi), available when M <= 512
+  int long_QV = 0;
+  uint32_t* d_long_msv = nullptr;
+  int32_t* d_long_rsc = nullptr;
+  int32_t* d_long_tr = nullptr;
   // threshold caches (built on first use per F and DB Lmax)
   std::mutex mu;
   struct Thr {
@@ -108,6 +126,8 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
 cudaError_t launch_msv_exact(const MsvArgs& a, int nwarps, cudaStream_t st);
 cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
+cudaError_t launch_pipe_long(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
+int long_msv_q(int QV);
 int msv_q_max(int G);
 int vit_q_max(int G);
 

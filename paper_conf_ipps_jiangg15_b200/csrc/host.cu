@@ -224,14 +224,14 @@ std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
   return t;
 }
 
-// Viterbi register-kernel tables: emissions as s16 pairs in the MSV chunk layout over Q2 words,
-// transitions as s32 [8][G*Q] with node (z*Q+q+1) at z*Q+q; nodes > M are -inf.
+// Viterbi register-kernel tables: emissions as s32 in the MSV chunk layout over Q words per lane
+// (lane z: nodes z*Q+1..z*Q+Q), transitions as s32 [8][G*Q] with node (z*Q+q+1) at z*Q+q;
+// nodes > M are -inf.
 void vit_tables(const hmg_profile& p, int G, int Q, std::vector<uint32_t>* rsc, std::vector<int32_t>* tr) {
   const int M = p.M;
-  const int Q2 = (Q + 1) / 2;
-  const int ROWW = Q2 * G;
+  const int ROWW = Q * G;
   rsc->assign(((size_t)kRows * ROWW + 3) / 4 * 4, 0);
-  const int n4 = Q2 / 4, r = Q2 % 4;
+  const int n4 = Q / 4, r = Q % 4;
   auto word_index = [&](int z, int q) {
     if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
     int b = n4 * 4 * G;
@@ -243,16 +243,12 @@ void vit_tables(const hmg_profile& p, int G, int Q, std::vector<uint32_t>* rsc, 
     }
     return b + z;
   };
-  auto r_of = [&](int x, int node) -> int16_t {
-    if (x >= kAlpha || node > M) return (int16_t)kNegW;
-    return p.rsc[(size_t)x * M + node - 1];
-  };
   for (int x = 0; x < kRows; ++x)
     for (int z = 0; z < G; ++z)
-      for (int h = 0; h < Q2; ++h) {
-        const uint16_t lo = (uint16_t)r_of(x, z * Q + 2 * h + 1);
-        const uint16_t hi = (2 * h + 1 < Q) ? (uint16_t)r_of(x, z * Q + 2 * h + 2) : (uint16_t)kNegW;
-        (*rsc)[(size_t)x * ROWW + word_index(z, h)] = (uint32_t)lo | ((uint32_t)hi << 16);
+      for (int q = 0; q < Q; ++q) {
+        const int node = z * Q + q + 1;
+        const int v = (x >= kAlpha || node > M) ? kNegW : (int)p.rsc[(size_t)x * M + node - 1];
+        (*rsc)[(size_t)x * ROWW + word_index(z, q)] = (uint32_t)v;
       }
   tr->assign((size_t)8 * G * Q, kNegW);
   for (int t = 0; t < 8; ++t)
@@ -341,19 +337,29 @@ MsvArgs msv_args(const hmg_profile* p, const hmg_db* db) {
   return a;
 }
 
-// MSV over the whole DB into raw_sorted (device, sorted order); fast kernel + exact redo.
-hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
+// number of leading (longest) sorted sequences with L > llong
+int64_t count_longer(const hmg_db* db, int llong) {
+  const auto it = std::upper_bound(db->len_sorted.begin(), db->len_sorted.end(), llong,
+                                   [](int v, int L) { return v > L; });
+  return (int64_t)(it - db->len_sorted.begin());
+}
+
+double mean_len(const hmg_db* db) { return db->nseq ? (double)db->residues / (double)db->nseq : 0.0; }
+
+// MSV fast kernel over the DB into raw_sorted (device, sorted order).  pipe_nlong >= 0: the
+// first pipe_nlong sequences are scored by the pipeline long lane instead.
+hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S,
+                        int64_t pipe_nlong) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
   a.raw = raw_sorted;
-  // long sequences: L > max(1000, 8 x mean length) (env HMG_MSV_LLONG overrides), length-sorted prefix
-  {
-    const double mean = n ? (double)db->residues / (double)n : 0.0;
-    const int llong = env_int("HMG_MSV_LLONG", (int)std::max(1000.0, 8.0 * mean));
-    const auto it = std::upper_bound(db->len_sorted.begin(), db->len_sorted.end(), llong,
-                                     [](int v, int L) { return v > L; });
-    a.nlong = (int64_t)(it - db->len_sorted.begin());
+  if (pipe_nlong >= 0) {
+    a.nlong = pipe_nlong;
+    a.skip_long = 1;
+  } else {  // in-kernel whole-warp queue: L > max(1000, 8 x mean length) (env HMG_MSV_LLONG)
+    a.nlong = count_longer(db, env_int("HMG_MSV_LLONG", (int)std::max(1000.0, 8.0 * mean_len(db))));
+    a.skip_long = 0;
   }
   auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
   if (e) return cuda_status(e);
@@ -366,7 +372,26 @@ hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint
     if ((e = launch_msv_fast(p->msv_G, p->msv_Q, a, st, &ok))) return cuda_status(e);
     if (!ok) return HMG_EUNSUPPORTED;
     mark(1, st);
-    // sequences whose every cell stayed <= B' are rescored exactly (rare)
+  } else {
+    auto* scr = (uint8_t*)S.get((size_t)nwarps_exact * 2 * (p->M + 1), &e);
+    if (e) return cuda_status(e);
+    a.list = nullptr;
+    a.scratch = scr;
+    mark(0, st);
+    if (n > 0 && (e = launch_msv_exact(a, nwarps_exact, st))) return cuda_status(e);
+    mark(1, st);
+  }
+  return HMG_OK;
+}
+
+// sequences the fast kernel flagged (every cell <= B') are rescored exactly (rare)
+hmg_status run_msv_redo(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
+  cudaError_t e = cudaSuccess;
+  const int64_t n = db->nseq;
+  if (p->msv_fast && p->msv_Q > 0) {
+    MsvArgs a = msv_args(p, db);
+    a.raw = raw_sorted;
+    const int nwarps_exact = 148 * 16;
     auto* list = (int32_t*)S.get(sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1), &e);
     auto* cnt = (int64_t*)S.get(sizeof(int64_t), &e);
     void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
@@ -377,23 +402,44 @@ hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint
     a.nlist = cnt;
     a.scratch = scr;
     if ((e = launch_msv_exact(a, nwarps_exact, st))) return cuda_status(e);
-    mark(2, st);
-  } else {
-    auto* scr = (uint8_t*)S.get((size_t)nwarps_exact * 2 * (p->M + 1), &e);
-    if (e) return cuda_status(e);
-    a.list = nullptr;
-    a.scratch = scr;
-    mark(0, st);
-    if (n > 0 && (e = launch_msv_exact(a, nwarps_exact, st))) return cuda_status(e);
-    mark(1, st);
-    mark(2, st);
   }
+  mark(2, st);
+  return HMG_OK;
+}
+
+hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
+  hmg_status s = run_msv_fast(p, db, st, raw_sorted, S, -1);
+  if (s != HMG_OK) return s;
+  return run_msv_redo(p, db, st, raw_sorted, S);
+}
+
+// per-device side stream + fork/join events for the pipeline long lane
+struct SideStream {
+  cudaStream_t s = nullptr;
+  cudaEvent_t fork = nullptr, join = nullptr;
+};
+SideStream g_side[64];
+std::mutex g_side_mu;
+
+hmg_status side_stream(int dev, SideStream** out) {
+  if (dev < 0 || dev >= 64) return HMG_EINVAL;
+  std::lock_guard<std::mutex> g(g_side_mu);
+  SideStream& S = g_side[dev];
+  if (!S.s) {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    cudaError_t e = cudaStreamCreateWithPriority(&S.s, cudaStreamNonBlocking, hi);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&S.fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&S.join, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_status(e);
+  }
+  *out = &S;
   return HMG_OK;
 }
 
 // Viterbi over sorted-order ids (list, device count) into raw_sorted.
 hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
-                   cudaStream_t st, int16_t* raw_sorted, Scratch& S) {
+                   cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr) {
   cudaError_t e = cudaSuccess;
   VitArgs a{};
   a.words = db->d_words;
@@ -407,6 +453,7 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
   a.list = list;
   a.nlist = nlist;
   a.raw_sorted = raw_sorted;
+  a.done = done;
   auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
@@ -595,6 +642,17 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       if (st == HMG_OK) st = upload(&p->d_tr, t.data(), t.size());
     }
   }
+  if (st == HMG_OK && tsc && M <= 512 && !env_int("HMG_NO_LONG_LANE", 0)) {
+    const int QV = (M + 31) / 32;
+    auto tm = msv_table(*p, 32, long_msv_q(QV));
+    std::vector<uint32_t> r;
+    std::vector<int32_t> t;
+    vit_tables(*p, 32, QV, &r, &t);
+    st = upload(&p->d_long_msv, tm.data(), tm.size());
+    if (st == HMG_OK) st = upload(reinterpret_cast<uint32_t**>(&p->d_long_rsc), r.data(), r.size());
+    if (st == HMG_OK) st = upload(&p->d_long_tr, t.data(), t.size());
+    if (st == HMG_OK) p->long_QV = QV;
+  }
   if (st != HMG_OK) {
     hmg_profile_destroy(p);
     return st;
@@ -634,6 +692,9 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_cost);
     cudaFree(p->d_rsc);
     cudaFree(p->d_tr);
+    cudaFree(p->d_long_msv);
+    cudaFree(p->d_long_rsc);
+    cudaFree(p->d_long_tr);
     cudaFree(p->thr_msv.d);
     cudaFree(p->thr_vit.d);
     cudaGetLastError();
@@ -876,12 +937,62 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
     if (e) return cuda_status(e);
     mark_reset();
-    s = run_msv(p, db, st, raw_sorted, S);                                   // Fig 1: MSV
+    // pipeline long lane (long.cu): the longest sequences get MSV + Viterbi on their own SMs,
+    // concurrently with the main MSV kernel (env HMG_PIPE_LLONG sets the length cut)
+    int64_t nlong = 0;
+    uint8_t* done = nullptr;
+    SideStream* side = nullptr;
+    if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && !p->vit_generic) {
+      nlong = count_longer(db, env_int("HMG_PIPE_LLONG", (int)std::max(1500.0, 8.0 * mean_len(db))));
+      if (nlong > 0 && (s = side_stream(db->device, &side)) != HMG_OK) return s;
+    }
+    if (nlong > 0) {
+      done = (uint8_t*)S.get((size_t)n, &e);
+      auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
+      if (e) return cuda_status(e);
+      if ((e = cudaMemsetAsync(done, 0, (size_t)n, st))) return cuda_status(e);
+      if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
+      LongArgs la{};
+      la.m = msv_args(p, db);
+      la.m.prof = p->d_long_msv;
+      la.m.raw = raw_sorted;
+      la.v.words = db->d_words;
+      la.v.woff16 = db->d_woff16;
+      la.v.len = db->d_len;
+      la.v.nseq = n;
+      la.v.move = db->d_move;
+      la.v.rsc = reinterpret_cast<const int16_t*>(p->d_long_rsc);
+      la.v.tr = p->d_long_tr;
+      la.v.M = p->M;
+      la.v.raw_sorted = vraw_sorted;
+      la.thr = tm;
+      la.done = done;
+      la.nlong = nlong;
+      la.counter = lctr;
+      // blocks (SMs) for the long lane: its row-cycles vs the main kernel's, with margin
+      int64_t rlong = 0;
+      for (int64_t j = 0; j < nlong; ++j) rlong += db->len_sorted[j];
+      const double main_cyc = (double)p->M * (double)(db->residues - rlong) / (55.0 * 140.0);
+      const double long_cyc = (double)rlong * 95.0 / 4.0;
+      int nb = (int)std::ceil(long_cyc / (0.6 * std::max(main_cyc, 1.0)));
+      nb = std::max(1, std::min(nb, std::min(32, (int)((nlong + 3) / 4))));
+      nb = env_int("HMG_PIPE_LONG_SMS", nb);
+      if ((e = cudaEventRecord(side->fork, st))) return cuda_status(e);
+      if ((e = cudaStreamWaitEvent(side->s, side->fork, 0))) return cuda_status(e);
+      int ok = 0;
+      if ((e = launch_pipe_long(p->long_QV, la, nb, side->s, &ok))) return cuda_status(e);
+      if (!ok) return HMG_EUNSUPPORTED;
+      if ((e = cudaEventRecord(side->join, side->s))) return cuda_status(e);
+    }
+    s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1);     // Fig 1: MSV
+    if (s != HMG_OK) return s;
+    if (nlong > 0 && (e = cudaStreamWaitEvent(st, side->join, 0))) return cuda_status(e);
+    s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;
     e = msv_finish(raw_sorted, db->d_len, db->d_order, n, tm, msv_raw, flags, surv, n_survivors, survivor_ids, tmp,
                    st);                                                       // pass + compaction
     if (e) return cuda_status(e);
-    s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S);               // P7Viterbi on survivors
+    s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S, done);         // P7Viterbi on survivors
     if (s != HMG_OK) return s;
     e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st);
     mark(5, st);

@@ -70,8 +70,8 @@ __device__ __forceinline__ int msv_thr(int xJ, int bias) {
 // Score one batch of 32/G sequences (sorted indices s0 + group) with G lanes per
 // sequence and Q s16x2 registers per lane, profile table `sm` in shared memory.
 template <int G, int Q>
-__device__ __forceinline__ void msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
-                                          long long send) {
+__device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
+                                         long long send) {
   constexpr int ROWW = Q * G;              // words per residue row
   const int lane = threadIdx.x & 31;
   const int z = lane & (G - 1);
@@ -151,13 +151,12 @@ __device__ __forceinline__ void msv_batch(const MsvArgs& a, const uint32_t* __re
 #pragma unroll
   for (int o = G / 2; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
   const int Rmax = max((int)(m & 0xffffu), (int)(m >> 16));
-  if (valid && z == 0) {
-    int raw;
-    if (ovf) raw = 255;
-    else if (Rmax > Bp) raw = max(xJ, max(Rmax - bias - 3, 0));
-    else raw = 254;                 // every cell <= B': exact kernel recomputes (rare)
-    a.raw[s] = (uint8_t)raw;
-  }
+  int raw;
+  if (ovf) raw = 255;
+  else if (Rmax > Bp) raw = max(xJ, max(Rmax - bias - 3, 0));
+  else raw = 254;                   // every cell <= B': exact kernel recomputes (rare)
+  if (valid && z == 0) a.raw[s] = (uint8_t)raw;
+  return raw;                       // identical on the G lanes of the group
 }
 
 // Long sequences (the first a.nlong in length order) use a whole warp (G = 32,
@@ -183,6 +182,7 @@ __global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
   const int lane = threadIdx.x & 31;
   if constexpr (QL > 0) {
     for (;;) {
+      if (a.skip_long) break;
       unsigned long long b = 0;
       if (lane == 0) b = atomicAdd(a.counter + 1, 1ull);
       b = __shfl_sync(0xffffffffu, b, 0);
@@ -191,7 +191,7 @@ __global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
     }
   }
   constexpr int NG = 32 / G;
-  const long long first = (QL > 0) ? a.nlong : 0;
+  const long long first = (QL > 0 || a.skip_long) ? a.nlong : 0;
   for (;;) {
     unsigned long long b = 0;
     if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);

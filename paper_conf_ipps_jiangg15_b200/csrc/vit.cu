@@ -33,8 +33,7 @@ cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int*
   const void* fn = vit_reg_ptr(G, Q);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
-  const int Q2 = (Q + 1) / 2;
-  const size_t smem = (((size_t)kRows * Q2 * G + 3) / 4) * 16;
+  const size_t smem = (((size_t)kRows * Q * G + 3) / 4) * 16;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = 0, per = 0;

@@ -30,38 +30,115 @@ namespace hmg {
 
 __device__ __forceinline__ int sadd(int a, int b) { return __viaddmax_s32(a, b, kNegW); }  // max(a+b, -32768)
 
+// One row of Alg 2 for the G-lane group (lane z owns nodes z*Q+1..z*Q+Q).
+// Returns nothing; updates Mc/Ic/Dc in place and the specials.
+template <int G, int Q>
+struct VitLane {
+  int tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
+  int Mc[Q], Ic[Q], Dc[Q];
+
+  __device__ __forceinline__ void row(const int32_t* __restrict__ rrow, int z, int& xB, int& xJ, int& xC,
+                                      int move, bool& ovf, bool live) {
+    int r[Q];
+    load_row<G, Q>(reinterpret_cast<const uint32_t*>(rrow), z, reinterpret_cast<uint32_t(&)[Q]>(r));
+    // diagonal carries: row i-1 values at node z*Q, owned by lane z-1 (none for lane 0)
+    int cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1, G);
+    int cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1, G);
+    int cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1, G);
+    if (z == 0) cM = cI = cD = kNegW;
+    // M and I (Alg 2 l.15-16), descending so that q-1 still holds row i-1
+#pragma unroll
+    for (int q = Q - 1; q >= 0; --q) {
+      const int pm = q ? Mc[q - 1] : cM;
+      const int pi = q ? Ic[q - 1] : cI;
+      const int pd = q ? Dc[q - 1] : cD;
+      int m = sadd(xB, tBM[q]);
+      m = __viaddmax_s32(pm, tMM[q], m);
+      m = __viaddmax_s32(pi, tIM[q], m);
+      m = __viaddmax_s32(pd, tDM[q], m);
+      Ic[q] = __viaddmax_s32(Ic[q], tII[q], sadd(Mc[q], tMI[q]));
+      Mc[q] = sadd(m, r[q]);                                  // + emission (reading R15)
+    }
+    int xE = kNegW;
+#pragma unroll
+    for (int q = 0; q + 1 < Q; q += 2) xE = __vimax3_s32(xE, Mc[q], Mc[q + 1]);
+    if constexpr (Q % 2) xE = max(xE, Mc[Q - 1]);
+    // D: partial from M (Alg 2 l.17, reading R16) fused with the in-lane D->D chain
+    Dc[0] = kNegW;
+#pragma unroll
+    for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], sadd(Mc[q - 1], tMD[q - 1]));
+    // xE over the group (Alg 2 l.22) and the specials (l.24; reading R17)
+    if constexpr (G == 32) {
+      xE = __reduce_max_sync(0xffffffffu, xE);
+    } else {
+#pragma unroll
+      for (int o = G / 2; o >= 1; o >>= 1) xE = max(xE, __shfl_xor_sync(0xffffffffu, xE, o));
+    }
+    if (live && !ovf) {
+      if (xE >= 32767) {
+        ovf = true;
+      } else {
+        xC = max(xC, xE - 500);
+        xJ = max(xJ, xE - 500);
+        xB = max(xJ, kBaseW) + move;
+      }
+    }
+    // Lazy-F across lane boundaries (l.25, Fig 7): each lane's outgoing D (+DD) feeds the
+    // next lane's first node; walk while it improves; repeat while any lane improved.
+    int cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], sadd(Mc[Q - 1], tMD[Q - 1]));
+    for (;;) {
+      int cin = __shfl_up_sync(0xffffffffu, cout, 1, G);
+      if (z == 0) cin = kNegW;
+      bool imp = cin > Dc[0];
+      if (!__any_sync(0xffffffffu, imp)) break;
+      Dc[0] = max(Dc[0], cin);
+      constexpr int K0 = Q < 3 ? Q : 3;      // most D->D runs die within a few nodes
+#pragma unroll
+      for (int q = 1; q < K0; ++q) {
+        const int nd = __viaddmax_s32(Dc[q - 1], tDD[q - 1], kNegW);
+        imp = imp && nd > Dc[q];
+        Dc[q] = max(Dc[q], nd);
+      }
+      if (__any_sync(0xffffffffu, imp)) {
+#pragma unroll
+        for (int q = K0; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], Dc[q]);
+        cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], cout);
+      } else {
+        break;
+      }
+    }
+  }
+};
+
 template <int G, int Q>
 __global__ void __launch_bounds__(128) vit_reg_kernel(const VitArgs a) {
-  constexpr int Q2 = (Q + 1) / 2;          // s16 emission pairs per lane
-  constexpr int ROWW = Q2 * G;             // words per residue row
+  constexpr int ROWW = Q * G;              // s32 words per residue row
   constexpr int NG = 32 / G;
   extern __shared__ uint4 smem4[];
-  uint32_t* sm = reinterpret_cast<uint32_t*>(smem4);
   {
     const uint4* src = reinterpret_cast<const uint4*>(a.rsc);
     const int n4 = (kRows * ROWW + 3) / 4;
     for (int i = threadIdx.x; i < n4; i += blockDim.x) smem4[i] = src[i];
   }
   __syncthreads();
+  const int32_t* sm = reinterpret_cast<const int32_t*>(smem4);
 
   const int lane = threadIdx.x & 31;
   const int z = lane & (G - 1);
   const int grp = lane / G;
-  const unsigned gbits = (G == 32 ? 0xffffffffu : ((1u << G) - 1u)) << (grp * G);
 
-  // this lane's transitions, s32, node k = z*Q + q + 1 (into-k: BM MM IM DM; out-of-k: MD MI II DD)
-  int tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
+  VitLane<G, Q> V;
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const int o = z * Q + q;
-    tBM[q] = a.tr[0 * G * Q + o];
-    tMM[q] = a.tr[1 * G * Q + o];
-    tIM[q] = a.tr[2 * G * Q + o];
-    tDM[q] = a.tr[3 * G * Q + o];
-    tMD[q] = a.tr[4 * G * Q + o];
-    tMI[q] = a.tr[5 * G * Q + o];
-    tII[q] = a.tr[6 * G * Q + o];
-    tDD[q] = a.tr[7 * G * Q + o];
+    const int o = z * Q + q;   // node z*Q + q + 1: into-k BM MM IM DM, out-of-k MD MI II DD
+    V.tBM[q] = a.tr[0 * G * Q + o];
+    V.tMM[q] = a.tr[1 * G * Q + o];
+    V.tIM[q] = a.tr[2 * G * Q + o];
+    V.tDM[q] = a.tr[3 * G * Q + o];
+    V.tMD[q] = a.tr[4 * G * Q + o];
+    V.tMI[q] = a.tr[5 * G * Q + o];
+    V.tII[q] = a.tr[6 * G * Q + o];
+    V.tDD[q] = a.tr[7 * G * Q + o];
   }
   const long long ntot = a.list ? *a.nlist : a.nseq;
 
@@ -71,8 +148,9 @@ __global__ void __launch_bounds__(128) vit_reg_kernel(const VitArgs a) {
     base = __shfl_sync(0xffffffffu, base, 0);
     if ((long long)base >= ntot) break;
     const long long idx = (long long)base + grp;
-    const bool valid = idx < ntot;
+    bool valid = idx < ntot;
     const int s = valid ? (a.list ? a.list[idx] : (int)idx) : 0;
+    if (valid && a.done && a.done[s]) valid = false;    // already scored by the pipeline long lane
     const int L = valid ? a.len[s] : 0;
     int Lmax = L;
 #pragma unroll
@@ -81,84 +159,20 @@ __global__ void __launch_bounds__(128) vit_reg_kernel(const VitArgs a) {
     const int nw = (L + 5) / 6;
     const int move = valid ? a.move[L] : 0;
 
-    int Mc[Q], Ic[Q], Dc[Q];
 #pragma unroll
-    for (int q = 0; q < Q; ++q) Mc[q] = Ic[q] = Dc[q] = kNegW;      // Alg 2 l.9
-    const int xN = kBaseW;
-    int xB = xN + move, xJ = kNegW, xC = kNegW;
-    bool ovf = false, done = !valid;
+    for (int q = 0; q < Q; ++q) V.Mc[q] = V.Ic[q] = V.Dc[q] = kNegW;      // Alg 2 l.9
+    int xB = kBaseW + move, xJ = kNegW, xC = kNegW;
+    bool ovf = false;
 
     const int nblk = (Lmax + 5) / 6;
     uint32_t wnext = (0 < nw) ? __ldg(wp) : 0xffffffffu;
     for (int blk = 0; blk < nblk; ++blk) {
       const uint32_t w = wnext;
       wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
-#pragma unroll 1
+#pragma unroll
       for (int j = 0; j < 6; ++j) {
-        const int x = (w >> (5 * j)) & 31;
-        if (x == kPadCode) done = true;                 // past the end of this sequence
-        uint32_t e2[Q2];
-        load_row<G, Q2>(sm + x * ROWW, z, e2);
-        // diagonal carries (row i-1 values at node z*Q, owned by lane z-1)
-        int cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1, G);
-        int cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1, G);
-        int cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1, G);
-        if (z == 0) cM = cI = cD = kNegW;
-        int xE = kNegW;
-        // M and I, descending so that q-1 still holds row i-1 (Alg 2 l.15-16)
-#pragma unroll
-        for (int q = Q - 1; q >= 0; --q) {
-          const int pm = q ? Mc[q - 1] : cM;
-          const int pi = q ? Ic[q - 1] : cI;
-          const int pd = q ? Dc[q - 1] : cD;
-          const int r = (q & 1) ? ((int)e2[q >> 1] >> 16) : (int)(int16_t)(e2[q >> 1] & 0xffffu);
-          int m = sadd(xB, tBM[q]);
-          m = __viaddmax_s32(pm, tMM[q], m);
-          m = __viaddmax_s32(pi, tIM[q], m);
-          m = __viaddmax_s32(pd, tDM[q], m);
-          m = sadd(m, r);                                       // + emission (reading R15)
-          const int in = __viaddmax_s32(Ic[q], tII[q], sadd(Mc[q], tMI[q]));
-          Mc[q] = m;
-          Ic[q] = in;
-        }
-#pragma unroll
-        for (int q = 0; q + 1 < Q; q += 2) xE = __vimax3_s32(xE, Mc[q], Mc[q + 1]);
-        if constexpr (Q % 2) xE = max(xE, Mc[Q - 1]);
-        // D: partial from M (Alg 2 l.17, reading R16) fused with the in-lane D->D chain
-        Dc[0] = kNegW;
-#pragma unroll
-        for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], sadd(Mc[q - 1], tMD[q - 1]));
-        // group max of xE (Alg 2 l.22)
-        if constexpr (G == 32) {
-          xE = __reduce_max_sync(0xffffffffu, xE);
-        } else {
-#pragma unroll
-          for (int o = G / 2; o >= 1; o >>= 1) xE = max(xE, __shfl_xor_sync(0xffffffffu, xE, o));
-        }
-        // specials (Alg 2 l.24; reading R17)
-        if (!done && !ovf) {
-          if (xE >= 32767) {
-            ovf = true;
-          } else {
-            xC = max(xC, xE - 500);
-            xJ = max(xJ, xE - 500);
-            xB = max(xJ, xN) + move;
-          }
-        }
-        // Lazy-F across lane boundaries (Alg 2 l.25; Fig 7)
-        int cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], sadd(Mc[Q - 1], tMD[Q - 1]));
-        for (;;) {
-          int cin = __shfl_up_sync(0xffffffffu, cout, 1, G);
-          if (z == 0) cin = kNegW;
-          const bool imp = cin > Dc[0];
-          if (!__any_sync(0xffffffffu, imp)) break;
-          if (imp) {
-            Dc[0] = cin;
-#pragma unroll
-            for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], Dc[q]);
-            cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], cout);
-          }
-        }
+        const int x = (w >> (5 * j)) & 31;          // 31: past the end of this sequence
+        V.row(sm + x * ROWW, z, xB, xJ, xC, move, ovf, x != kPadCode);
       }
     }
     if (valid && z == 0) a.raw_sorted[s] = (int16_t)(ovf ? 32767 : xC);
