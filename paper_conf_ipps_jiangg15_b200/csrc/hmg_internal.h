@@ -54,18 +54,24 @@ struct VitArgs {
   int16_t* raw_sorted;       // [nseq] output, sorted order
   unsigned long long* counter;
   int32_t* scratch;          // generic kernel: per-warp rows
-  const uint8_t* done;       // register kernel: skip sorted index s when done[s] (long lane ran it)
+  const uint8_t* done;       // skip sorted index s < ndone when done[s] (the pipeline long lane owns it)
+  int64_t ndone;
 };
 
-// Pipeline long lane: MSV (whole warp) then, on pass, Viterbi (whole warp) for the
-// longest sequences, on SMs it holds exclusively, concurrently with the main MSV kernel.
+// Pipeline long lane (long.cu): chunked whole-warp MSV for the longest sequences, then
+// whole-warp Viterbi for their MSV survivors on SMs held alone, concurrent with the main MSV.
 struct LongArgs {
   MsvArgs m;                 // m.prof = whole-warp MSV table (32, QL), m.raw = MSV raw (sorted)
   VitArgs v;                 // v.rsc / v.tr = register-kernel tables (32, QV), v.raw_sorted
   const uint16_t* thr;       // MSV pass threshold by length
-  uint8_t* done;             // [nseq] set to 1 where the Viterbi filter ran here
+  uint8_t* owned;            // [nlong] 1: the long lane runs the Viterbi filter of this sequence
   int64_t nlong;
-  unsigned long long* counter;
+  const int32_t* chunk_start;  // [nlong+1] exclusive prefix of row chunks per long sequence
+  int64_t nitems;            // total chunks
+  int chunk_rows;
+  int* chunk_max;            // [nitems]
+  unsigned* chunk_done;      // [nlong] chunks finished
+  unsigned long long* counter;  // [2] work queues (chunks, Viterbi)
 };
 
 }  // namespace hmg
@@ -82,6 +88,7 @@ struct hmg_profile {
   hmg_evparams ev{};
   int msv_fast = 0, msv_G = 0, msv_Q = 0;
   int vit_G = 0, vit_Q = 0, vit_generic = 0;
+  int vit_W = 0;                    // >0: block-per-sequence kernel vit_cta_kernel<W, Q> (Q = vit_Q)
   // device tables
   uint32_t* d_msv_prof = nullptr;   // striped s16x2 emissions
   uint8_t* d_cost = nullptr;        // [kRows][M]
@@ -117,6 +124,12 @@ struct hmg_db {
   uint8_t* d_tjb = nullptr;       // [Lmax+1]
   int16_t* d_move = nullptr;      // [Lmax+1]
   std::vector<uint32_t> host_image;  // host-only handles (device < 0)
+  // pipeline long lane: sequences [0, nlong) with L > long_cut, cut into chunk_rows-row chunks
+  int long_cut = 0;
+  int64_t nlong = 0;
+  int chunk_rows = 1032;
+  int64_t nchunks = 0;
+  int32_t* d_chunk_start = nullptr;  // [nlong+1]
 };
 
 namespace hmg {
@@ -126,7 +139,10 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
 cudaError_t launch_msv_exact(const MsvArgs& a, int nwarps, cudaStream_t st);
 cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
-cudaError_t launch_pipe_long(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
+cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
+cudaError_t launch_vit_cta(int W, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+size_t vit_cta_smem(int W, int Q);
 int long_msv_q(int QV);
 int msv_q_max(int G);
 int vit_q_max(int G);

@@ -166,7 +166,8 @@ int env_int(const char* name, int dflt) {
 
 // ---------------------------------------------------------------- kernel geometry
 void msv_geometry(int M, int* G, int* Q) {
-  int g = M <= 128 ? 4 : M <= 512 ? 8 : M <= 1024 ? 16 : 32;
+  // lane-group size from the G sweep on the config-2 DB (profiles/msv_sweep_r01.txt)
+  int g = M < 80 ? 8 : M <= 640 ? 16 : 32;
   const int o = env_int("HMG_MSV_G", 0);
   if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
   // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
@@ -254,6 +255,40 @@ void vit_tables(const hmg_profile& p, int G, int Q, std::vector<uint32_t>* rsc, 
   for (int t = 0; t < 8; ++t)
     for (int o = 0; o < G * Q; ++o)
       if (o < M) (*tr)[(size_t)t * G * Q + o] = p.tsc[(size_t)t * M + o];
+}
+
+// block-per-sequence kernel tables: emissions as s16 pairs (node g*Q+2h+1 low, +2 high) in the
+// chunk layout over Q/2 words per lane; transitions as vit_tables.
+void vit_tables_s16(const hmg_profile& p, int NT, int Q, std::vector<uint32_t>* rsc, std::vector<int32_t>* tr) {
+  const int M = p.M;
+  const int Q2 = Q / 2;
+  const int ROWW = Q2 * NT;
+  rsc->assign((size_t)kRows * ROWW, 0);
+  const int n4 = Q2 / 4, r = Q2 % 4;
+  auto word_index = [&](int z, int q) {
+    if (q < n4 * 4) return (q / 4) * 4 * NT + z * 4 + (q % 4);
+    int b = n4 * 4 * NT;
+    int qq = q - n4 * 4;
+    if (r >= 2) {
+      if (qq < 2) return b + z * 2 + qq;
+      b += 2 * NT;
+      qq -= 2;
+    }
+    return b + z;
+  };
+  auto r_of = [&](int x, int node) -> uint16_t {
+    if (x >= kAlpha || node > M) return (uint16_t)(int16_t)kNegW;
+    return (uint16_t)p.rsc[(size_t)x * M + node - 1];
+  };
+  for (int x = 0; x < kRows; ++x)
+    for (int z = 0; z < NT; ++z)
+      for (int h = 0; h < Q2; ++h)
+        (*rsc)[(size_t)x * ROWW + word_index(z, h)] =
+            (uint32_t)r_of(x, z * Q + 2 * h + 1) | ((uint32_t)r_of(x, z * Q + 2 * h + 2) << 16);
+  tr->assign((size_t)8 * NT * Q, kNegW);
+  for (int t = 0; t < 8; ++t)
+    for (int o = 0; o < NT * Q; ++o)
+      if (o < M) (*tr)[(size_t)t * NT * Q + o] = p.tsc[(size_t)t * M + o];
 }
 
 struct Scratch {
@@ -439,7 +474,8 @@ hmg_status side_stream(int dev, SideStream** out) {
 
 // Viterbi over sorted-order ids (list, device count) into raw_sorted.
 hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
-                   cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr) {
+                   cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr,
+                   int64_t ndone = 0) {
   cudaError_t e = cudaSuccess;
   VitArgs a{};
   a.words = db->d_words;
@@ -454,12 +490,17 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
   a.nlist = nlist;
   a.raw_sorted = raw_sorted;
   a.done = done;
+  a.ndone = done ? ndone : 0;
   auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
   a.counter = ctr;
   mark(3, st);
-  if (!p->vit_generic) {
+  if (!p->vit_generic && p->vit_W > 0) {
+    int ok = 0;
+    if ((e = launch_vit_cta(p->vit_W, p->vit_Q, a, st, &ok))) return cuda_status(e);
+    if (!ok) return HMG_EUNSUPPORTED;
+  } else if (!p->vit_generic) {
     int ok = 0;
     if ((e = launch_vit_reg(p->vit_G, p->vit_Q, a, st, &ok))) return cuda_status(e);
     if (!ok) return HMG_EUNSUPPORTED;
@@ -602,6 +643,21 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   msv_geometry(M, &p->msv_G, &p->msv_Q);
   if (tsc) {
     vit_geometry(M, &p->vit_G, &p->vit_Q);
+    if (p->vit_Q == 0 || env_int("HMG_VIT_CTA", 0)) {   // long models: block-per-sequence kernel
+      const int W = M <= 1024 ? 8 : 16;
+      int Q = (M + 32 * W - 1) / (32 * W);
+      Q += Q & 1;
+      int smax = 0;   // the s16 emission table must fit in one block's shared memory
+      if (device >= 0) cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+      else smax = 227 * 1024;
+      if (Q <= 8 && vit_cta_smem(W, Q) <= (size_t)smax) {
+        p->vit_W = W;
+        p->vit_G = 32 * W;
+        p->vit_Q = Q;
+      } else {
+        p->vit_Q = 0;
+      }
+    }
     p->vit_generic = p->vit_Q == 0 || env_int("HMG_VIT_GENERIC", 0);
   }
   if (device < 0) {
@@ -626,7 +682,15 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     st = upload(&p->d_msv_prof, t.data(), t.size());
   }
   if (st == HMG_OK && tsc) {
-    if (!p->vit_generic) {
+    if (!p->vit_generic && p->vit_W > 0) {
+      std::vector<uint32_t> r;
+      std::vector<int32_t> t;
+      vit_tables_s16(*p, p->vit_G, p->vit_Q, &r, &t);
+      p->vit_rsc_bytes = r.size() * 4;
+      p->vit_tr_bytes = t.size() * 4;
+      st = upload(reinterpret_cast<uint32_t**>(&p->d_rsc), r.data(), r.size());
+      if (st == HMG_OK) st = upload(&p->d_tr, t.data(), t.size());
+    } else if (!p->vit_generic) {
       std::vector<uint32_t> r;
       std::vector<int32_t> t;
       vit_tables(*p, p->vit_G, p->vit_Q, &r, &t);
@@ -679,7 +743,7 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->msv_fast = p->msv_fast;
   q->msv_lanes = p->msv_G;
   q->msv_regs = p->msv_Q;
-  q->vit_lanes = p->vit_generic ? 32 : p->vit_G;
+  q->vit_lanes = p->vit_generic ? 32 : p->vit_G;   // block kernel: 32 * warps
   q->vit_nodes = p->vit_generic ? 0 : p->vit_Q;
   return HMG_OK;
 }
@@ -775,6 +839,19 @@ hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, i
   }
   std::vector<int32_t> inv(nseq);
   for (int64_t j = 0; j < nseq; ++j) inv[db->order[j]] = (int32_t)j;
+  // pipeline long lane: L > max(1500, 8 x mean) (env HMG_PIPE_LLONG), chunks of 1032 rows
+  std::vector<int32_t> cstart(1, 0);
+  {
+    const double mean = nseq ? (double)res / (double)nseq : 0.0;
+    db->long_cut = env_int("HMG_PIPE_LLONG", (int)std::max(1500.0, 8.0 * mean));
+    db->chunk_rows = std::max(6, env_int("HMG_PIPE_CHUNK", 1032) / 6 * 6);
+    while (db->nlong < nseq && db->len_sorted[db->nlong] > db->long_cut) {
+      const int L = db->len_sorted[db->nlong];
+      cstart.push_back(cstart.back() + (L + db->chunk_rows - 1) / db->chunk_rows);
+      ++db->nlong;
+    }
+    db->nchunks = cstart.back();
+  }
   if (device < 0) {
     db->host_image = std::move(img);
     *out = db;
@@ -788,6 +865,7 @@ hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, i
   if (st == HMG_OK) st = upload(&db->d_inv, inv.data(), inv.size());
   if (st == HMG_OK) st = upload(&db->d_tjb, tjb.data(), tjb.size());
   if (st == HMG_OK) st = upload(&db->d_move, mv.data(), mv.size());
+  if (st == HMG_OK) st = upload(&db->d_chunk_start, cstart.data(), cstart.size());
   if (st != HMG_OK) {
     hmg_db_destroy(db);
     return st;
@@ -834,6 +912,7 @@ void hmg_db_destroy(hmg_db* db) {
     cudaFree(db->d_inv);
     cudaFree(db->d_tjb);
     cudaFree(db->d_move);
+    cudaFree(db->d_chunk_start);
     cudaGetLastError();
   }
   delete db;
@@ -937,21 +1016,21 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
     if (e) return cuda_status(e);
     mark_reset();
-    // pipeline long lane (long.cu): the longest sequences get MSV + Viterbi on their own SMs,
-    // concurrently with the main MSV kernel (env HMG_PIPE_LLONG sets the length cut)
-    int64_t nlong = 0;
-    uint8_t* done = nullptr;
+    // pipeline long lane (long.cu): chunked whole-warp MSV of the longest sequences, then their
+    // Viterbi on SMs held alone (side stream) while the main MSV kernel runs on the others
+    const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && !p->vit_generic && p->vit_W == 0 &&
+                           !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
+    uint8_t* owned = nullptr;
     SideStream* side = nullptr;
-    if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && !p->vit_generic) {
-      nlong = count_longer(db, env_int("HMG_PIPE_LLONG", (int)std::max(1500.0, 8.0 * mean_len(db))));
-      if (nlong > 0 && (s = side_stream(db->device, &side)) != HMG_OK) return s;
-    }
     if (nlong > 0) {
-      done = (uint8_t*)S.get((size_t)n, &e);
-      auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
+      if ((s = side_stream(db->device, &side)) != HMG_OK) return s;
+      owned = (uint8_t*)S.get((size_t)nlong, &e);
+      auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+      auto* cmax = (int*)S.get(sizeof(int) * (size_t)std::max<int64_t>(db->nchunks, 1), &e);
+      auto* cdone = (unsigned*)S.get(sizeof(unsigned) * (size_t)nlong, &e);
       if (e) return cuda_status(e);
-      if ((e = cudaMemsetAsync(done, 0, (size_t)n, st))) return cuda_status(e);
-      if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
+      if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+      if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * (size_t)nlong, st))) return cuda_status(e);
       LongArgs la{};
       la.m = msv_args(p, db);
       la.m.prof = p->d_long_msv;
@@ -966,34 +1045,35 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       la.v.M = p->M;
       la.v.raw_sorted = vraw_sorted;
       la.thr = tm;
-      la.done = done;
+      la.owned = owned;
       la.nlong = nlong;
+      la.chunk_start = db->d_chunk_start;
+      la.nitems = db->nchunks;
+      la.chunk_rows = db->chunk_rows;
+      la.chunk_max = cmax;
+      la.chunk_done = cdone;
       la.counter = lctr;
-      // blocks (SMs) for the long lane: its row-cycles vs the main kernel's, with margin
-      int64_t rlong = 0;
-      for (int64_t j = 0; j < nlong; ++j) rlong += db->len_sorted[j];
-      const double main_cyc = (double)p->M * (double)(db->residues - rlong) / (55.0 * 140.0);
-      const double long_cyc = (double)rlong * 95.0 / 4.0;
-      int nb = (int)std::ceil(long_cyc / (0.6 * std::max(main_cyc, 1.0)));
-      nb = std::max(1, std::min(nb, std::min(32, (int)((nlong + 3) / 4))));
+      int ok = 0;
+      if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);   // main stream
+      if (!ok) return HMG_EUNSUPPORTED;
+      // Viterbi of the long survivors on a side stream, on SMs held alone
+      int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
       nb = env_int("HMG_PIPE_LONG_SMS", nb);
       if ((e = cudaEventRecord(side->fork, st))) return cuda_status(e);
       if ((e = cudaStreamWaitEvent(side->s, side->fork, 0))) return cuda_status(e);
-      int ok = 0;
-      if ((e = launch_pipe_long(p->long_QV, la, nb, side->s, &ok))) return cuda_status(e);
-      if (!ok) return HMG_EUNSUPPORTED;
+      if ((e = launch_pipe_long_vit(p->long_QV, la, nb, side->s, &ok))) return cuda_status(e);
       if ((e = cudaEventRecord(side->join, side->s))) return cuda_status(e);
     }
     s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1);     // Fig 1: MSV
     if (s != HMG_OK) return s;
-    if (nlong > 0 && (e = cudaStreamWaitEvent(st, side->join, 0))) return cuda_status(e);
     s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;
     e = msv_finish(raw_sorted, db->d_len, db->d_order, n, tm, msv_raw, flags, surv, n_survivors, survivor_ids, tmp,
                    st);                                                       // pass + compaction
     if (e) return cuda_status(e);
-    s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S, done);         // P7Viterbi on survivors
+    s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S, owned, nlong);  // P7Viterbi on survivors
     if (s != HMG_OK) return s;
+    if (nlong > 0 && (e = cudaStreamWaitEvent(st, side->join, 0))) return cuda_status(e);
     e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st);
     mark(5, st);
   }

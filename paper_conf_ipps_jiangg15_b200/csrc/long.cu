@@ -1,15 +1,20 @@
-// long.cu -- the pipeline's long lane: whole-warp MSV then Viterbi for the longest sequences.
+// long.cu -- the pipeline's long lane: the longest sequences (L > ~8x the mean length).
 //
 // A DP row cannot be split across time (Alg 1/2 carry xB from row i to i+1), so a
 // sequence's filter time is bounded below by its length times the row latency of one
-// lane group.  On a B200 the warp arbiter shares issue slots evenly among resident
-// warps (measured: profiles/arbiter_r01.txt), so a long sequence sharing its SM
-// sub-partition with five other warps runs five to six times slower than alone.
-// The longest sequences (L > ~8x the mean) therefore run here: one warp per
-// sequence, 4 warps per block, each block asking for enough shared memory to hold
-// its SM alone, MSV with G = 32 (msv_batch<32, QL>) and -- if the MSV pass flag is
-// set -- the Viterbi filter right away (VitLane<32, QV>).  The main MSV kernel runs
-// concurrently on the remaining SMs; the Viterbi kernel later skips what ran here.
+// lane group; and the B200 warp arbiter shares issue slots evenly among resident warps
+// (measured, profiles/arbiter_r01.txt), so a long sequence sharing its SM sub-partition
+// with five other warps runs five to six times slower than alone.  Two kernels:
+//
+// pipe_long_msv_kernel<QL>: MSV of the long sequences cut into row chunks that run in
+//   parallel, each from the empty state M rows early (exact: an MSV domain is one ungapped
+//   diagonal, so row i depends only on rows > i - M while xB is unchanged).  The last
+//   chunk of a sequence to finish combines the chunk maxima; if any chunk saw a row that
+//   could move xB (a hit) or overflow, it re-runs the sequence with the sequential
+//   whole-warp DP (msv_batch<32, QL>).  It runs on the main stream before the main MSV.
+// pipe_long_vit_kernel<QV>: Viterbi filter (whole warp, latency variant of VitLane) of the
+//   long MSV survivors, longest first, on SMs it holds alone (each block asks for most of
+//   the shared memory), concurrently with the main MSV kernel on the other SMs.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -23,89 +28,164 @@ namespace hmg {
 __host__ __device__ constexpr int long_msv_q_of(int QV) { return (32 * QV + 1 + 63) / 64; }
 int long_msv_q(int QV) { return long_msv_q_of(QV); }
 
-template <int QV>
-__global__ void __launch_bounds__(128) pipe_long_kernel(const LongArgs A) {
-  constexpr int QL = long_msv_q_of(QV);
-  constexpr int WM = kRows * QL * 32;       // MSV table words
-  constexpr int WV = kRows * QV * 32;       // Viterbi emission table words
+template <int QL>
+__global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
+  constexpr int WM = kRows * QL * 32;
   extern __shared__ uint4 smem4[];
   {
     const uint4* s0 = reinterpret_cast<const uint4*>(A.m.prof);
     for (int i = threadIdx.x; i < WM / 4; i += blockDim.x) smem4[i] = s0[i];
-    const uint4* s1 = reinterpret_cast<const uint4*>(A.v.rsc);
-    for (int i = threadIdx.x; i < WV / 4; i += blockDim.x) smem4[WM / 4 + i] = s1[i];
   }
   __syncthreads();
   const uint32_t* smm = reinterpret_cast<const uint32_t*>(smem4);
-  const int32_t* smv = reinterpret_cast<const int32_t*>(smem4) + WM;
   const int lane = threadIdx.x & 31;
-
-  VitLane<32, QV> V;
-#pragma unroll
-  for (int q = 0; q < QV; ++q) {
-    const int o = lane * QV + q;
-    V.tBM[q] = A.v.tr[0 * 32 * QV + o];
-    V.tMM[q] = A.v.tr[1 * 32 * QV + o];
-    V.tIM[q] = A.v.tr[2 * 32 * QV + o];
-    V.tDM[q] = A.v.tr[3 * 32 * QV + o];
-    V.tMD[q] = A.v.tr[4 * 32 * QV + o];
-    V.tMI[q] = A.v.tr[5 * 32 * QV + o];
-    V.tII[q] = A.v.tr[6 * 32 * QV + o];
-    V.tDD[q] = A.v.tr[7 * 32 * QV + o];
-  }
   for (;;) {
     unsigned long long b = 0;
     if (lane == 0) b = atomicAdd(A.counter, 1ull);
     b = __shfl_sync(0xffffffffu, b, 0);
+    if ((long long)b >= A.nitems) break;
+    // item -> (sequence j, chunk c): chunk_start is the exclusive prefix of chunks per sequence
+    int lo = 0, hi = (int)A.nlong;             // largest j with chunk_start[j] <= b
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if ((unsigned long long)A.chunk_start[mid] <= b) lo = mid;
+      else hi = mid;
+    }
+    const int j = lo;
+    const int c = (int)(b - A.chunk_start[j]);
+    const int nch = A.chunk_start[j + 1] - A.chunk_start[j];
+    const int L = A.m.len[j];
+    const int r0 = c * A.chunk_rows;
+    const int r1 = min(L, r0 + A.chunk_rows);
+    int rm = 0;
+    const bool ok = msv_chunk<QL>(A.m, smm, j, r0, r1, A.m.M, &rm);
+    if (lane == 0) {
+      A.chunk_max[b] = ok ? rm : -1;
+      __threadfence();
+    }
+    unsigned prev = 0;
+    if (lane == 0) prev = atomicAdd(A.chunk_done + j, 1u);
+    prev = __shfl_sync(0xffffffffu, prev, 0);
+    if ((int)prev != nch - 1) continue;          // not the last chunk of sequence j
+    __threadfence();
+    // last finisher: combine, or fall back to the sequential DP
+    int Rmax = 0;
+    bool all_ok = true;
+    for (int k = A.chunk_start[j] + lane; k < A.chunk_start[j + 1]; k += 32) {
+      const int v = *((volatile int*)A.chunk_max + k);
+      if (v < 0) all_ok = false;
+      Rmax = max(Rmax, v);
+    }
+    all_ok = __all_sync(0xffffffffu, all_ok);
+    Rmax = __reduce_max_sync(0xffffffffu, Rmax);
+    int raw;
+    if (all_ok) {
+      const int tjb = A.m.tjb[L];
+      const int Bp = min(max(kBaseB - tjb - A.m.tbm, 0) + A.m.bias, 255);
+      raw = Rmax > Bp ? max(Rmax - A.m.bias - 3, 0) : 254;
+      if (lane == 0) A.m.raw[j] = (uint8_t)raw;
+    } else {
+      raw = msv_batch<32, QL>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
+    }
+    if (lane == 0) A.owned[j] = raw != 254;     // 254: exact re-score on the main stream decides
+  }
+}
+
+template <int QV>
+__global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
+  constexpr int WV = kRows * QV * 32;        // Viterbi emission table words
+  extern __shared__ uint4 smem4[];
+  {
+    const uint4* s1 = reinterpret_cast<const uint4*>(A.v.rsc);
+    for (int i = threadIdx.x; i < WV / 4; i += blockDim.x) smem4[i] = s1[i];
+  }
+  __syncthreads();
+  const int32_t* smv = reinterpret_cast<const int32_t*>(smem4);
+  const int lane = threadIdx.x & 31;
+  VitLane<32, QV, true> V;
+  V.load(A.v.tr, lane);
+  for (;;) {
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(A.counter + 1, 1ull);
+    b = __shfl_sync(0xffffffffu, b, 0);
     if ((long long)b >= A.nlong) break;
     const int s = (int)b;
-    const int raw = msv_batch<32, QL>(A.m, smm, (long long)s, A.nlong);   // Alg 1
+    if (!A.owned[s]) continue;
+    const int raw = A.m.raw[s];
     const int L = A.m.len[s];
-    const bool pass = raw == 255 || (raw != 254 && raw >= (int)A.thr[L]);
-    if (!pass) continue;                      // 254: the exact MSV re-scores it; main stage decides
-    // Alg 2 on this survivor, same warp, right away
+    if (!(raw == 255 || raw >= (int)A.thr[L])) continue;       // MSV pass flag (reading R25)
     const uint32_t* wp = A.v.words + (size_t)A.v.woff16[s] * 4;
     const int nw = (L + 5) / 6;
-    const int move = A.v.move[L];
+    V.start(A.v.move[L], true);
+    ResStream rs;
+    rs.init(wp, nw);
+    for (int iq = 0; iq < rs.nq; ++iq) {                        // Alg 2 row loop
+      uint4 w4 = rs.next(iq);
+#pragma unroll 1
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t w = w4.x;
+        w4.x = w4.y;
+        w4.y = w4.z;
+        w4.z = w4.w;
 #pragma unroll
-    for (int q = 0; q < QV; ++q) V.Mc[q] = V.Ic[q] = V.Dc[q] = kNegW;
-    int xB = kBaseW + move, xJ = kNegW, xC = kNegW;
-    bool ovf = false;
-    uint32_t wnext = __ldg(wp);
-    for (int blk = 0; blk < nw; ++blk) {
-      const uint32_t w = wnext;
-      wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
-#pragma unroll
-      for (int j = 0; j < 6; ++j) {
-        const int x = (w >> (5 * j)) & 31;
-        V.row(smv + x * (QV * 32), lane, xB, xJ, xC, move, ovf, x != kPadCode);
+        for (int j = 0; j < 6; ++j) {
+          const int x = (w >> (5 * j)) & 31;
+          V.row(smv + x * (QV * 32), lane, 0xffffffffu);
+        }
       }
     }
-    if (lane == 0) {
-      A.v.raw_sorted[s] = (int16_t)(ovf ? 32767 : xC);
-      A.done[s] = 1;
-    }
+    const int vraw = V.finish();
+    if (lane == 0) A.v.raw_sorted[s] = (int16_t)vraw;
   }
 }
 
 namespace {
 template <int QV>
-const void* pick(int q) {
+const void* pick_vit(int q) {
   if constexpr (QV > 16) {
     return nullptr;
   } else {
-    if (q == QV) return reinterpret_cast<const void*>(&pipe_long_kernel<QV>);
-    return pick<QV + 1>(q);
+    if (q == QV) return reinterpret_cast<const void*>(&pipe_long_vit_kernel<QV>);
+    return pick_vit<QV + 1>(q);
+  }
+}
+template <int QL>
+const void* pick_msv(int q) {
+  if constexpr (QL > 8) {
+    return nullptr;
+  } else {
+    if (q == QL) return reinterpret_cast<const void*>(&pipe_long_msv_kernel<QL>);
+    return pick_msv<QL + 1>(q);
   }
 }
 }  // namespace
 
-cudaError_t launch_pipe_long(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
-  const void* fn = pick<1>(QV);
+cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int* ok) {
+  const int QL = long_msv_q_of(QV);
+  const void* fn = pick_msv<1>(QL);
+  *ok = fn != nullptr;
+  if (!fn) return cudaSuccess;
+  const size_t smem = (size_t)kRows * QL * 32 * 4;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, nsm = 0, per = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, 256, smem);
+  if (e != cudaSuccess) return e;
+  const int64_t need = (a.nitems + 7) / 8;
+  int64_t grid = std::min<int64_t>((int64_t)nsm * std::max(per, 1), std::max<int64_t>(need, 1));
+  void* args[] = {const_cast<LongArgs*>(&a)};
+  g_launches += 1;
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args, smem, st);
+}
+
+cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
+  const void* fn = pick_vit<1>(QV);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
   // ask for most of the SM's shared memory so no block of another kernel shares the SM
-  const size_t need = ((size_t)kRows * long_msv_q_of(QV) * 32 + (size_t)kRows * QV * 32) * 4;
+  const size_t need = (size_t)kRows * QV * 32 * 4;
   int dev = 0, maxsm = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);

@@ -60,6 +60,28 @@ __device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z
   }
 }
 
+// Residue stream of one sequence: 16-byte quads of packed words (24 residues) fetched two
+// quads ahead, so the DRAM/L2 latency of the residue stream hides behind >= 24 DP rows even
+// for short models.  Words past the sequence are all-31 (pad rows).
+struct ResStream {
+  const uint4* p;
+  int nq;
+  uint4 cur, nxt;
+  __device__ __forceinline__ static uint4 pad() { return make_uint4(~0u, ~0u, ~0u, ~0u); }
+  __device__ __forceinline__ void init(const uint32_t* wp, int nw) {
+    p = reinterpret_cast<const uint4*>(wp);
+    nq = (nw + 3) / 4;
+    cur = nq > 0 ? __ldg(p) : pad();
+    nxt = nq > 1 ? __ldg(p + 1) : pad();
+  }
+  __device__ __forceinline__ uint4 next(int iq) {   // quad iq, prefetching iq + 2
+    const uint4 r = cur;
+    cur = nxt;
+    nxt = (iq + 2 < nq) ? __ldg(p + iq + 2) : pad();
+    return r;
+  }
+};
+
 __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
   int T = max(xJ, 189) + 4;
@@ -101,11 +123,17 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
   for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
   uint32_t R = B2;
 
-  const int nblk = (Lmax + 5) / 6;
-  uint32_t wnext = (0 < nw) ? __ldg(wp) : 0xffffffffu;
-  for (int blk = 0; blk < nblk; ++blk) {
-    const uint32_t w = wnext;
-    wnext = (blk + 1 < nw) ? __ldg(wp + blk + 1) : 0xffffffffu;
+  const int nqmax = (Lmax + 23) / 24;
+  ResStream rs;
+  rs.init(wp, nw);
+  for (int iq = 0; iq < nqmax; ++iq) {
+   uint4 w4 = rs.next(iq);
+#pragma unroll 1
+   for (int k = 0; k < 4; ++k) {
+    const uint32_t w = w4.x;
+    w4.x = w4.y;
+    w4.y = w4.z;
+    w4.z = w4.w;
 #pragma unroll
     for (int j = 0; j < 6; ++j) {
       const int x = (w >> (5 * j)) & 31;
@@ -145,6 +173,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
         }
       }
     }
+   }
   }
   // final xJ = max over all cells of (s - 3); R holds max over t = max(s + bias, B')
   uint32_t m = R;
@@ -157,6 +186,64 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
   else raw = 254;                   // every cell <= B': exact kernel recomputes (rare)
   if (valid && z == 0) a.raw[s] = (uint8_t)raw;
   return raw;                       // identical on the G lanes of the group
+}
+
+// Rows [r0, r1) of one sequence with a whole warp, starting from the empty state (t = B')
+// `warm` rows earlier.  Exact for rows >= r0 whenever warm >= M - 1 and xB stays at its initial
+// value: an MSV path is one ungapped diagonal segment per domain, so a cell of row i only
+// depends on rows > i - M.  Returns false if a counted row reached the J->B /
+// overflow threshold (xB would change: the caller falls back to the sequential DP);
+// otherwise *rmax = max t over the counted rows.
+template <int Q>
+__device__ __forceinline__ bool msv_chunk(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s, int r0,
+                                          int r1, int warm, int* rmax) {
+  constexpr int G = 32;
+  constexpr int ROWW = Q * G;
+  const int z = threadIdx.x & 31;
+  const uint32_t sel = (z == 0) ? 0x1054u : 0x3210u;
+  const uint32_t negpair = (uint32_t)(uint16_t)kNegE;
+  const int bias = a.bias, tbm = a.tbm;
+  const int L = a.len[s];
+  const uint32_t* wp = a.words + (size_t)a.woff16[s] * 4;
+  const int nw = (L + 5) / 6;
+  const int tjb = a.tjb[L];
+  const int Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
+  const uint32_t B2 = (uint32_t)Bp * 0x10001u;
+  const uint32_t thrv = (uint32_t)(0x8000 - msv_thr(0, bias)) * 0x10001u;
+  uint32_t t[Q];
+#pragma unroll
+  for (int q = 0; q < Q; ++q) t[q] = B2;
+  uint32_t R = B2;
+  const int wc = r0 / 6;                       // first counted word (r0 is a multiple of 6)
+  const int wb = max(0, r0 - warm) / 6;        // first warm-up word
+  const int we = min(nw, (r1 + 5) / 6);
+  for (int blk = wb; blk < we; ++blk) {
+    const uint32_t w = __ldg(wp + blk);
+    const bool counting = blk >= wc;
+#pragma unroll
+    for (int j = 0; j < 6; ++j) {
+      const int x = (w >> (5 * j)) & 31;
+      uint32_t e[Q];
+      load_row<G, Q>(sm + x * ROWW, z, e);
+      uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
+      c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
+      c = __byte_perm(c, negpair, sel);
+#pragma unroll
+      for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
+      t[0] = __vmaxs2(c, B2);
+      if (counting) {
+#pragma unroll
+        for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
+        if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+        if (__any_sync(0xffffffffu, (__vadd2(R, thrv) & 0x80008000u) != 0u)) return false;
+      }
+    }
+  }
+  uint32_t m = R;
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) m = __vmaxs2(m, __shfl_xor_sync(0xffffffffu, m, o));
+  *rmax = max((int)(m & 0xffffu), (int)(m >> 16));
+  return true;
 }
 
 // Long sequences (the first a.nlong in length order) use a whole warp (G = 32,

@@ -312,3 +312,40 @@ def test_msv_config2_full_size_sampled():
                                        np.argsort(db.lengths)[:40]]))
     want = oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off, ids=sample)
     assert np.array_equal(got[sample], want)
+
+
+@pytest.mark.parametrize("M", [2, 3, 64, 255, 300, 513, 700, 1024, 1025, 1500, 2048, 2600, 4000])
+@pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
+def test_vit_block_kernel(M, dd, monkeypatch):
+    """Block-per-sequence Viterbi (W warps per row, cross-warp Lazy-F through shared memory);
+    forced for small M with HMG_VIT_CTA, used by default above M = 512."""
+    monkeypatch.setenv("HMG_VIT_CTA", "1")
+    rng = np.random.default_rng(M * 3 + int(dd[1]))
+    prof = synth.make_profile(M, 9000 + M, dd=dd)
+    n = 30 if M <= 1100 else 10
+    dsq, off = _ragged_db(rng, n=n, alphabet=29, lmax=250)
+    got, p = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+    q = p.quant()
+    assert q["vit_lanes"] >= 256 or M > 3072       # beyond: general kernel (table > 227 KB)
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off))
+
+
+@pytest.mark.parametrize("M", [40, 300, 700, 2000])
+def test_vit_block_kernel_delete_chains(M, monkeypatch):
+    """D->D chains that cross every warp boundary of the block (cross-warp Lazy-F rounds)."""
+    monkeypatch.setenv("HMG_VIT_CTA", "1")
+    rng = np.random.default_rng(M + 5)
+    msc = np.full((M, 29), -6.0, np.float32)
+    msc[0, 0] = 4.0
+    msc[M - 1, 1] = 4.0
+    msc[M // 2, 2] = 3.0
+    tsc = np.log(rng.uniform(0.05, 1.0, size=(M, 8))).astype(np.float32)
+    tsc[:, 7] = np.log(rng.uniform(0.9, 0.9999, size=M))
+    tsc[1:, 0] = -np.inf
+    tsc[0, 1:4] = -np.inf
+    tsc[M - 1, 4:8] = -np.inf
+    seqs = [np.array([0, 1], np.uint8), np.array([0, 2, 1], np.uint8), np.array([0, 1, 0, 2, 1], np.uint8)]
+    seqs += [synth.random_dsq(rng, int(L), 3) for L in rng.integers(1, 40, size=12)]
+    dsq, off = _db_from(seqs)
+    got, _ = _vit_gpu(msc, tsc, dsq, off)
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
