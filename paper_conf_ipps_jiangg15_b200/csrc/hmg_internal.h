@@ -71,6 +71,7 @@ struct LongArgs {
   int chunk_rows;
   int* chunk_max;            // [nitems]
   unsigned* chunk_done;      // [nlong] chunks finished
+  unsigned* ready;           // [nlong] 1 once the MSV raw / owned flag of the sequence are final
   unsigned long long* counter;  // [2] work queues (chunks, Viterbi)
 };
 

@@ -167,7 +167,7 @@ int env_int(const char* name, int dflt) {
 // ---------------------------------------------------------------- kernel geometry
 void msv_geometry(int M, int* G, int* Q) {
   // lane-group size from the G sweep on the config-2 DB (profiles/msv_sweep_r01.txt)
-  int g = M < 80 ? 8 : M <= 640 ? 16 : 32;
+  int g = M < 80 ? 8 : M < 150 ? 16 : M <= 450 ? 8 : M <= 640 ? 16 : 32;
   const int o = env_int("HMG_MSV_G", 0);
   if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
   // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
@@ -442,10 +442,53 @@ hmg_status run_msv_redo(const hmg_profile* p, const hmg_db* db, cudaStream_t st,
   return HMG_OK;
 }
 
+hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted,
+                               Scratch& S, LongArgs* la_out);
+
+// MSV over the whole DB: the longest sequences as parallel row chunks (long.cu), the rest with
+// the lane-group kernel; then the exact re-score of flagged sequences.
 hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
-  hmg_status s = run_msv_fast(p, db, st, raw_sorted, S, -1);
+  int64_t nlong = -1;
+  if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && db->nlong > 0 && !env_int("HMG_NO_LONG_LANE", 0)) {
+    LongArgs la{};
+    hmg_status s = run_msv_long_chunks(p, db, st, raw_sorted, S, &la);
+    if (s != HMG_OK) return s;
+    nlong = db->nlong;
+  }
+  hmg_status s = run_msv_fast(p, db, st, raw_sorted, S, nlong);
   if (s != HMG_OK) return s;
   return run_msv_redo(p, db, st, raw_sorted, S);
+}
+
+// set up the long-lane arguments (scratch on S) and launch the chunked MSV on st
+hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted,
+                               Scratch& S, LongArgs* la_out) {
+  cudaError_t e = cudaSuccess;
+  const int64_t nlong = db->nlong;
+  auto* owned = (uint8_t*)S.get((size_t)nlong, &e);
+  auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+  auto* cmax = (int*)S.get(sizeof(int) * (size_t)std::max<int64_t>(db->nchunks, 1), &e);
+  auto* cdone = (unsigned*)S.get(sizeof(unsigned) * 2 * (size_t)nlong, &e);   // chunk_done | ready
+  if (e) return cuda_status(e);
+  if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+  if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * 2 * (size_t)nlong, st))) return cuda_status(e);
+  LongArgs& la = *la_out;
+  la = LongArgs{};
+  la.m = msv_args(p, db);
+  la.m.prof = p->d_long_msv;
+  la.m.raw = raw_sorted;
+  la.owned = owned;
+  la.nlong = nlong;
+  la.chunk_start = db->d_chunk_start;
+  la.nitems = db->nchunks;
+  la.chunk_rows = db->chunk_rows;
+  la.chunk_max = cmax;
+  la.chunk_done = cdone;
+  la.ready = cdone + nlong;
+  la.counter = lctr;
+  int ok = 0;
+  if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
+  return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 
 // per-device side stream + fork/join events for the pipeline long lane
@@ -644,7 +687,9 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   if (tsc) {
     vit_geometry(M, &p->vit_G, &p->vit_Q);
     if (p->vit_Q == 0 || env_int("HMG_VIT_CTA", 0)) {   // long models: block-per-sequence kernel
-      const int W = M <= 1024 ? 8 : 16;
+      int W = M <= 2048 ? 8 : 16;           // W = 8 keeps two 256-thread blocks per SM up to M = 2048
+      const int wo = env_int("HMG_VIT_CTA_W", 0);
+      if (wo == 4 || wo == 8 || wo == 16) W = wo;
       int Q = (M + 32 * W - 1) / (32 * W);
       Q += Q & 1;
       int smax = 0;   // the s16 emission table must fit in one block's shared memory
@@ -1027,10 +1072,10 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       owned = (uint8_t*)S.get((size_t)nlong, &e);
       auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
       auto* cmax = (int*)S.get(sizeof(int) * (size_t)std::max<int64_t>(db->nchunks, 1), &e);
-      auto* cdone = (unsigned*)S.get(sizeof(unsigned) * (size_t)nlong, &e);
+      auto* cdone = (unsigned*)S.get(sizeof(unsigned) * 2 * (size_t)nlong, &e);   // chunk_done | ready
       if (e) return cuda_status(e);
       if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
-      if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * (size_t)nlong, st))) return cuda_status(e);
+      if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * 2 * (size_t)nlong, st))) return cuda_status(e);
       LongArgs la{};
       la.m = msv_args(p, db);
       la.m.prof = p->d_long_msv;
@@ -1052,17 +1097,28 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       la.chunk_rows = db->chunk_rows;
       la.chunk_max = cmax;
       la.chunk_done = cdone;
+      la.ready = cdone + nlong;
       la.counter = lctr;
+      // Viterbi of the long survivors on a side stream, on SMs held alone.  It is enqueued
+      // first so its blocks are placed before the main MSV kernel fills the GPU, and it waits
+      // per sequence (ready[]) for the chunked MSV below, which runs on the other SMs.
       int ok = 0;
-      if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);   // main stream
-      if (!ok) return HMG_EUNSUPPORTED;
-      // Viterbi of the long survivors on a side stream, on SMs held alone
       int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
       nb = env_int("HMG_PIPE_LONG_SMS", nb);
+      const bool sync_mode = env_int("HMG_LONG_SYNC", 0) != 0;   // diagnostics: no overlap
+      if (sync_mode) {
+        if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
+        if (!ok) return HMG_EUNSUPPORTED;
+      }
       if ((e = cudaEventRecord(side->fork, st))) return cuda_status(e);
       if ((e = cudaStreamWaitEvent(side->s, side->fork, 0))) return cuda_status(e);
       if ((e = launch_pipe_long_vit(p->long_QV, la, nb, side->s, &ok))) return cuda_status(e);
+      if (!ok) return HMG_EUNSUPPORTED;
       if ((e = cudaEventRecord(side->join, side->s))) return cuda_status(e);
+      if (!sync_mode) {
+        if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);   // main stream
+        if (!ok) return HMG_EUNSUPPORTED;
+      }
     }
     s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1);     // Fig 1: MSV
     if (s != HMG_OK) return s;

@@ -87,7 +87,11 @@ __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
     } else {
       raw = msv_batch<32, QL>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
     }
-    if (lane == 0) A.owned[j] = raw != 254;     // 254: exact re-score on the main stream decides
+    if (lane == 0) {
+      A.owned[j] = raw != 254;                  // 254: exact re-score on the main stream decides
+      __threadfence();
+      atomicExch(A.ready + j, 1u);              // publish to pipe_long_vit_kernel
+    }
   }
 }
 
@@ -110,8 +114,15 @@ __global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
     b = __shfl_sync(0xffffffffu, b, 0);
     if ((long long)b >= A.nlong) break;
     const int s = (int)b;
-    if (!A.owned[s]) continue;
-    const int raw = A.m.raw[s];
+    // wait until the MSV of sequence s is final (pipe_long_msv_kernel runs concurrently on the
+    // other SMs and finishes the longest sequences first)
+    if (lane == 0) {
+      while (atomicAdd(A.ready + s, 0u) == 0u) __nanosleep(256);
+      __threadfence();
+    }
+    __syncwarp();
+    if (!*((volatile uint8_t*)A.owned + s)) continue;
+    const int raw = *((volatile uint8_t*)A.m.raw + s);
     const int L = A.m.len[s];
     if (!(raw == 255 || raw >= (int)A.thr[L])) continue;       // MSV pass flag (reading R25)
     const uint32_t* wp = A.v.words + (size_t)A.v.woff16[s] * 4;
@@ -151,7 +162,7 @@ const void* pick_vit(int q) {
 }
 template <int QL>
 const void* pick_msv(int q) {
-  if constexpr (QL > 8) {
+  if constexpr (QL > 9) {   // QV <= 16 -> QL <= 9
     return nullptr;
   } else {
     if (q == QL) return reinterpret_cast<const void*>(&pipe_long_msv_kernel<QL>);
@@ -182,8 +193,16 @@ cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int
 
 cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
   const void* fn = pick_vit<1>(QV);
-  *ok = fn != nullptr;
-  if (!fn) return cudaSuccess;
+  const void* producer = pick_msv<1>(long_msv_q_of(QV));
+  *ok = fn != nullptr && producer != nullptr;
+  if (!*ok) return cudaSuccess;
+  // This kernel spins on flags the chunked-MSV kernel sets.  With CUDA's lazy module loading the
+  // first launch of a kernel may synchronise the context, which would wait on this spinning
+  // kernel forever: force both kernels to be loaded before this one is launched.
+  cudaFuncAttributes fa;
+  cudaError_t e0 = cudaFuncGetAttributes(&fa, producer);
+  if (e0 == cudaSuccess) e0 = cudaFuncGetAttributes(&fa, fn);
+  if (e0 != cudaSuccess) return e0;
   // ask for most of the SM's shared memory so no block of another kernel shares the SM
   const size_t need = (size_t)kRows * QV * 32 * 4;
   int dev = 0, maxsm = 0;
@@ -191,6 +210,9 @@ cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStr
   cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   const size_t smem = std::max(need, (size_t)maxsm - 8192);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const size_t psmem = (size_t)kRows * long_msv_q_of(QV) * 32 * 4;
+  e = cudaFuncSetAttribute(producer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem);
   if (e != cudaSuccess) return e;
   void* args[] = {const_cast<LongArgs*>(&a)};
   g_launches += 1;

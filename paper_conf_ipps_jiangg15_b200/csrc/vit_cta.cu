@@ -24,7 +24,10 @@ const void* pick(int W, int Q) {
 }
 }  // namespace
 
-size_t vit_cta_smem(int W, int Q) { return (size_t)kRows * (Q / 2) * 32 * W * 4 + (2 * W * 3 + 2 * W + W) * 4; }
+size_t vit_cta_smem(int W, int Q) {
+  // VitCtaSmem<W, Q>::table_bytes + NSCR ints
+  return (size_t)21 * (Q / 2) * 32 * W * 4 + (size_t)(8 * W + 2 * W + 5 * W + 1) * 4;
+}
 
 cudaError_t launch_vit_cta(int W, int Q, const VitArgs& a, cudaStream_t st, int* ok) {
   const void* fn = pick(W, Q);

@@ -2,16 +2,24 @@
 //
 // For long models (M up to 32*W*Q, e.g. 2048 with W = 16 warps x Q = 4 nodes) and for the
 // latency-bound longest sequences, W warps cooperate on one DP row: thread g = 32*w + lane
-// owns the contiguous nodes g*Q+1 .. g*Q+Q with its 8 transition vectors and M/I/D cells in
-// registers (as in vit_reg_kernel).  Per row, besides the intra-warp shuffles:
-//   * diagonal carries across warp boundaries: lane 31 of warp w-1 publishes its (M, I, D)
-//     for the next row in shared memory (double-buffered by row parity);
-//   * Lazy-F across warps (Fig 7): every warp first closes D inside itself, then
-//     publishes its outgoing carry; each warp applies its neighbour's carry; rounds repeat
-//     while __syncthreads_or says some warp's outgoing carry improved (reading R19);
-//   * hits: the running-max xE vote of vit.cuh becomes __syncthreads_or; on a hit row the
-//     block reduces xE through shared memory and recomputes the B->M terms.
-// Emission scores are s16 pairs in shared memory (32 rows x M x 2 B: 128 KB at M = 2048).
+// owns the contiguous nodes g*Q+1 .. g*Q+Q with its transition vectors and M/I/D cells in
+// registers, as in vit_reg_kernel.  ONE block barrier per row:
+//
+//   D->D (Lazy-F, Fig 7) is resolved as a max-plus carry chain.  Each thread's
+//   block of nodes maps an incoming D carry c to an outgoing max(cl, c + bsum), where cl is
+//   the outgoing carry computed directly from its M cells (max_q M_q + tMD_q + later tDD) and
+//   bsum the sum of its tDD.  Inside a warp the incoming carries are found by shuffles
+//   repeated while __any_sync reports a change (reading R19); across warps each warp
+//   publishes its outgoing carry, and after the barrier every warp folds the carries of the
+//   warps to its left itself (W <= 16 steps), so no further barrier round is needed.  With
+//   sat(a + t) = max(a + t, -32768) and t <= 0 this is the same fixed point as the oracle's
+//   sequential closure.
+//   Diagonal carries across warp boundaries (row i-1 values at node 32*w*Q) are rebuilt by the
+//   right-hand warp from the ingredients lane 31 of the left warp published before the barrier.
+//   Hits (a row whose best M cell may move xB) are detected by the running-max vote of vit.cuh
+//   folded into the same barrier (__syncthreads_or); only then is xE reduced over the block.
+// Emission scores are s16 pairs; the 20 canonical rows and X live in shared memory (21 x M x 2 B:
+// 86 KB at M = 2048, two blocks per SM), the rare codes (B J Z O U, gaps) are read from L2.
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -25,12 +33,17 @@ struct VitCtaSmem {
   static constexpr int NT = 32 * W;          // threads = lanes of the DP row
   static constexpr int Q2 = Q / 2;           // s16 emission pairs per lane
   static constexpr int ROWW = Q2 * NT;       // u32 words per residue row
-  static constexpr size_t table_bytes = (size_t)kRows * ROWW * 4;
-  // shared scratch after the table (ints)
-  static constexpr int XC = 0;               // [2][W][3] diagonal carries (M, I, D of lane 31)
-  static constexpr int WC = XC + 2 * W * 3;  // [2][W] outgoing D carry of each warp
-  static constexpr int RX = WC + 2 * W;      // [W] per-warp xE max on hit rows
-  static constexpr int NSCR = RX + W;
+  static constexpr int SROWS = 21;           // shared rows: 20 canonical residues + X (code 26)
+  static constexpr size_t table_bytes = (size_t)SROWS * ROWW * 4;
+  // int scratch after the table
+  static constexpr int XC = 0;               // [2][W][4]  lane 31: M, I, D (in-thread), carry into it
+  static constexpr int WO = XC + 2 * W * 4;  // [2][W]     warp outgoing D carry (warp incoming = -inf)
+  static constexpr int BW = WO + 2 * W;      // [W]        sum of tDD over the warp's nodes
+  static constexpr int P31 = BW + W;         // [W]        lane 31: prefix of bsum inside the warp
+  static constexpr int S31 = P31 + W;        // [W]        lane 31: prefix of tDD to its last node
+  static constexpr int RX = S31 + W;         // [W]        per-warp xE max on hit rows
+  static constexpr int PB = RX + W;          // [W+1]      exclusive prefix of BW over the warps
+  static constexpr int NSCR = PB + W + 1;
 };
 
 template <int W, int Q>
@@ -40,7 +53,9 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
   extern __shared__ uint4 smem4[];
   {
     const uint4* src = reinterpret_cast<const uint4*>(a.rsc);
-    for (int i = threadIdx.x; i < (int)(S::table_bytes / 16); i += blockDim.x) smem4[i] = src[i];
+    constexpr int R16 = S::ROWW / 4;           // uint4 per row
+    for (int i = threadIdx.x; i < 20 * R16; i += blockDim.x) smem4[i] = src[i];
+    for (int i = threadIdx.x; i < R16; i += blockDim.x) smem4[20 * R16 + i] = src[26 * R16 + i];
   }
   uint32_t* tab = reinterpret_cast<uint32_t*>(smem4);
   int* scr = reinterpret_cast<int*>(reinterpret_cast<char*>(smem4) + S::table_bytes);
@@ -50,6 +65,7 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
 
   // transitions of this thread's nodes (into-k BM MM IM DM, out-of-k MD MI II DD), s32
   int tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
+  int ps[Q], wout[Q];
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     const int o = g * Q + q;
@@ -57,7 +73,47 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
     tBM[q] = a.tr[0 * NQ + o]; tMM[q] = a.tr[1 * NQ + o]; tIM[q] = a.tr[2 * NQ + o]; tDM[q] = a.tr[3 * NQ + o];
     tMD[q] = a.tr[4 * NQ + o]; tMI[q] = a.tr[5 * NQ + o]; tII[q] = a.tr[6 * NQ + o]; tDD[q] = a.tr[7 * NQ + o];
   }
+  int bsum = 0;
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    ps[q] = bsum;                            // sum of tDD before node q inside the thread
+    bsum += tDD[q];
+  }
+  {
+    int acc = 0;
+#pragma unroll
+    for (int q = Q - 1; q >= 0; --q) {
+      wout[q] = tMD[q] + acc;                // M_q -> D_{q+1} -> ... -> next thread's first node
+      acc += tDD[q];
+    }
+  }
+  // exclusive prefix of bsum over the lanes of the warp (constant), and warp totals
+  int pbs = bsum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, pbs, o);
+    if (lane >= o) pbs += y;
+  }
+  pbs -= bsum;
+  if (lane == 31) {
+    scr[S::BW + w] = pbs + bsum;
+    scr[S::P31 + w] = pbs;
+    scr[S::S31 + w] = ps[Q - 1];
+  }
   __syncthreads();
+  if (g == 0) {
+    int acc = 0;
+    for (int v = 0; v < W; ++v) {
+      scr[S::PB + v] = acc;
+      acc += scr[S::BW + v];
+    }
+    scr[S::PB + W] = acc;
+  }
+  __syncthreads();
+  // carry into warp w from warps v < w: PB[w] + max_v (WO[v] - PB[v+1]); lane v holds PB[v+1]
+  const int pb_next = lane < W ? scr[S::PB + lane + 1] : 0;
+  const int pb_w = scr[S::PB + w];
+  const int pb_wl = w > 0 ? scr[S::PB + w - 1] : 0;
   const long long ntot = a.list ? *a.nlist : a.nseq;
 
   for (;;) {
@@ -80,38 +136,38 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
     int R = kNegW, xJ = kNegW;
     bool ovf = false;
     int thr = min(kBaseW + 501, 32767);
-    if (lane == 31) {
-      scr[S::XC + (0 * W + w) * 3 + 0] = kNegW;
-      scr[S::XC + (0 * W + w) * 3 + 1] = kNegW;
-      scr[S::XC + (0 * W + w) * 3 + 2] = kNegW;
-    }
-    __syncthreads();
-    int par = 0;                               // row parity (buffer holding row i-1's carries)
+    // row -1 (all -inf) as seen from the right-hand warp
+    int nbM = kNegW, nbI = kNegW, nbD = kNegW;
+    int par = 0;
+    uint32_t wcur = __ldg(wp), wnxt = L > 6 ? __ldg(wp + 1) : ~0u;
     for (int i = 0; i < L; ++i) {
-      const int x = (__ldg(wp + i / 6) >> (5 * (i % 6))) & 31;
-      // emissions (s16 pairs -> s32)
+      const int j6 = i % 6;
+      const int x = (wcur >> (5 * j6)) & 31;
+      if (j6 == 5) {                              // next word; prefetch the one after it
+        wcur = wnxt;
+        wnxt = (i / 6 + 2) * 6 < L ? __ldg(wp + i / 6 + 2) : ~0u;
+      }
+      const uint32_t* rowp = x < 20 ? tab + x * S::ROWW
+                                    : (x == 26 ? tab + 20 * S::ROWW
+                                               : reinterpret_cast<const uint32_t*>(a.rsc) + x * S::ROWW);
       uint32_t e2[S::Q2];
-      load_row<S::NT, S::Q2>(tab + x * S::ROWW, g, e2);
+      load_row<S::NT, S::Q2>(rowp, g, e2);
       int r[Q];
 #pragma unroll
       for (int h = 0; h < S::Q2; ++h) {
         r[2 * h] = (int)(int16_t)(e2[h] & 0xffffu);
         r[2 * h + 1] = (int)e2[h] >> 16;
       }
-      // diagonal carries (row i-1 at node g*Q): lane l-1, or lane 31 of warp w-1
+      // diagonal carries (row i-1 at node g*Q): lane l-1, or lane 31 of warp w-1 (nb*)
       int cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
       int cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
       int cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
       if (lane == 0) {
-        if (w == 0) {
-          cM = cI = cD = kNegW;
-        } else {
-          const int* xc = scr + S::XC + (par * W + (w - 1)) * 3;
-          cM = xc[0];
-          cI = xc[1];
-          cD = xc[2];
-        }
+        cM = nbM;
+        cI = nbI;
+        cD = nbD;
       }
+      // M and I (Alg 2 l.15-16, emission per reading R15)
 #pragma unroll
       for (int q = Q - 1; q >= 0; --q) {
         const int pm = q ? Mc[q - 1] : cM;
@@ -125,28 +181,50 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
       }
 #pragma unroll
       for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s32(R, Mc[q], Mc[q + 1]);
-      // D partial (l.17) + in-thread D->D chain
+      // D partial (l.17) + in-thread chain, and this thread's outgoing carry from its M cells
+      int cl = kNegW;
+#pragma unroll
+      for (int q = 0; q < Q; ++q) cl = __viaddmax_s32(Mc[q], wout[q], cl);
       Dc[0] = kNegW;
 #pragma unroll
       for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], sadd(Mc[q - 1], tMD[q - 1]));
-      int cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], sadd(Mc[Q - 1], tMD[Q - 1]));
-      // intra-warp Lazy-F with the warp's incoming carry taken as -inf (applied below)
+      // carries inside the warp: ci = outgoing of lane-1, iterate while any lane changes
+      int out = cl, ci;
       for (;;) {
-        int cin = __shfl_up_sync(0xffffffffu, cout, 1);
-        if (lane == 0) cin = kNegW;
-        bool imp = cin > Dc[0];
-        if (!__any_sync(0xffffffffu, imp)) break;
-        if (imp) {
-          Dc[0] = cin;
-#pragma unroll
-          for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], Dc[q]);
-          cout = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], cout);
-        }
+        ci = __shfl_up_sync(0xffffffffu, out, 1);
+        if (lane == 0) ci = kNegW;
+        const int o2 = max(cl, __viaddmax_s32(ci, bsum, kNegW));
+        const bool chg = o2 != out;
+        out = o2;
+        if (!__any_sync(0xffffffffu, chg)) break;
       }
-      int rnd = 0;
-      if (lane == 31) scr[S::WC + (rnd & 1) * W + w] = cout;
-      // hit / overflow (running max, reading R17) joins the first block barrier
+      const int wr = par * W + w;
+      if (lane == 31) {
+        scr[S::WO + wr] = out;                       // warp outgoing (warp incoming = -inf)
+        scr[S::XC + wr * 4 + 0] = Mc[Q - 1];
+        scr[S::XC + wr * 4 + 1] = Ic[Q - 1];
+        scr[S::XC + wr * 4 + 2] = Dc[Q - 1];           // in-thread D of the last node (pre-carry)
+        scr[S::XC + wr * 4 + 3] = ci;                  // intra-warp carry into lane 31
+      }
+      // the row's one barrier; hit / overflow vote folded in (reading R17)
       const bool hit = __syncthreads_or(R >= thr);
+      // carries from the warps on the left: cw = into this warp, cwl = into warp w-1
+      const int av = lane < W ? scr[S::WO + par * W + lane] - pb_next : kNegW * 64;
+      const int m1 = __reduce_max_sync(0xffffffffu, lane < w ? av : kNegW * 64);
+      const int m2 = __reduce_max_sync(0xffffffffu, lane + 1 < w ? av : kNegW * 64);
+      const int cw = w > 0 ? max(kNegW, pb_w + m1) : kNegW;
+      const int cwl = w > 1 ? max(kNegW, pb_wl + m2) : kNegW;
+      const int cf = max(ci, __viaddmax_s32(cw, pbs, kNegW));    // final carry into this thread
+#pragma unroll
+      for (int q = 0; q < Q; ++q) Dc[q] = __viaddmax_s32(cf, ps[q], Dc[q]);
+      // next row's diagonal carry for lane 0: warp w-1's last node, rebuilt here
+      if (w > 0 && lane == 0) {
+        const int* xc = scr + S::XC + (par * W + w - 1) * 4;
+        const int cf31 = max(xc[3], __viaddmax_s32(cwl, scr[S::P31 + w - 1], kNegW));
+        nbM = xc[0];
+        nbI = xc[1];
+        nbD = __viaddmax_s32(cf31, scr[S::S31 + w - 1], xc[2]);
+      }
       if (hit) {
         int m = __reduce_max_sync(0xffffffffu, R);
         if (lane == 0) scr[S::RX + w] = m;
@@ -154,6 +232,7 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
         m = kNegW;
 #pragma unroll
         for (int v = 0; v < W; ++v) m = max(m, scr[S::RX + v]);
+        __syncthreads();
         if (!ovf) {
           if (m >= 32767) {
             ovf = true;
@@ -166,37 +245,6 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
             thr = min(max(xJ, kBaseW) + 501, 32767);
           }
         }
-      }
-      // Lazy-F across warps: apply the left neighbour's outgoing carry, repeat while it changes
-      for (;;) {
-        int cin = (w > 0) ? scr[S::WC + (rnd & 1) * W + (w - 1)] : kNegW;
-        cin = __shfl_sync(0xffffffffu, cin, 0);
-        bool changed = false;
-        const bool imp = (lane == 0) && cin > Dc[0];
-        if (__any_sync(0xffffffffu, imp)) {
-          if (imp) Dc[0] = cin;
-          for (;;) {                                  // propagate inside the warp
-#pragma unroll
-            for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], Dc[q]);
-            const int c2 = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], cout);
-            int cn = __shfl_up_sync(0xffffffffu, c2, 1);
-            const bool more = lane > 0 && cn > Dc[0];
-            if (more) Dc[0] = cn;
-            const bool lane_changed = c2 > cout;
-            cout = c2;
-            if (lane == 31 && lane_changed) changed = true;
-            if (!__any_sync(0xffffffffu, more)) break;
-          }
-        }
-        ++rnd;
-        if (lane == 31) {
-          scr[S::WC + (rnd & 1) * W + w] = cout;
-          const int np = par ^ 1;
-          scr[S::XC + (np * W + w) * 3 + 0] = Mc[Q - 1];
-          scr[S::XC + (np * W + w) * 3 + 1] = Ic[Q - 1];
-          scr[S::XC + (np * W + w) * 3 + 2] = Dc[Q - 1];
-        }
-        if (!__syncthreads_or(changed)) break;
       }
       par ^= 1;
     }

@@ -130,6 +130,7 @@ class Profile:
                                         ctypes.byref(evp) if evp is not None else None, device, ctypes.byref(h)),
                "hmg_profile_create")
         self._h = h
+        self._destroy = lib().hmg_profile_destroy
         self.device = device
 
     @property
@@ -148,7 +149,7 @@ class Profile:
 
     def close(self):
         if getattr(self, "_h", None):
-            lib().hmg_profile_destroy(self._h)
+            self._destroy(self._h)
             self._h = None
 
     __del__ = close
@@ -166,6 +167,7 @@ class Database:
         _check(lib().hmg_db_create(_np_ptr(dsq) if len(dsq) else None, _np_ptr(off), self.nseq, device,
                                    ctypes.byref(h)), "hmg_db_create")
         self._h = h
+        self._destroy = lib().hmg_db_destroy
         self.device = device
         self.lengths = np.diff(off).astype(np.int32)
 
@@ -203,7 +205,7 @@ class Database:
 
     def close(self):
         if getattr(self, "_h", None):
-            lib().hmg_db_destroy(self._h)
+            self._destroy(self._h)
             self._h = None
 
     __del__ = close

@@ -349,3 +349,26 @@ def test_vit_block_kernel_delete_chains(M, monkeypatch):
     dsq, off = _db_from(seqs)
     got, _ = _vit_gpu(msc, tsc, dsq, off)
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
+
+
+@pytest.mark.parametrize("chunk", [1032, 60])
+def test_pipeline_long_lane(chunk, monkeypatch):
+    """The pipeline long lane: sequences longer than max(1500, 8 x mean) get chunked MSV (rows
+    from the empty state M rows early) and whole-warp Viterbi on a side stream.  Strong planted
+    hits in some long sequences force the sequential fallback (a chunk sees a J->B row)."""
+    monkeypatch.setenv("HMG_PIPE_CHUNK", str(chunk))
+    rng = np.random.default_rng(42)
+    prof = synth.make_profile(120, 4242)
+    best = np.argmax(prof.msc[:, :20], axis=1).astype(np.uint8)
+    seqs = []
+    for i in range(300):
+        L = int(rng.integers(1600, 7000)) if i < 40 else int(rng.integers(20, 400))
+        d = synth.random_dsq(rng, L, 20)
+        if i % 5 == 0:                      # plant a strong hit somewhere
+            seg = best[: min(len(best), L)]
+            a = int(rng.integers(0, L - len(seg) + 1))
+            d[a:a + len(seg)] = seg
+        seqs.append(d)
+    dsq, off = _db_from(seqs)
+    ns = _check_pipeline(prof, dsq, off, F1=0.02, F2=1e-3)
+    assert ns >= 10
