@@ -115,6 +115,11 @@ int64_t hmg_db_nseq(const hmg_db* db);
 int64_t hmg_db_residues(const hmg_db* db);
 int64_t hmg_db_packed_bytes(const hmg_db* db);   /* size of the packed residue image */
 
+/* Long-sequence lane of this DB: the number of sequences (the longest, L > max(1500, 8 x mean
+ * length)) that hmg_msv / hmg_pipeline score as parallel row chunks and, in the pipeline, on
+ * SMs of their own; *residues (may be NULL) receives their residue count. */
+int64_t hmg_db_long_lane(const hmg_db* db, int64_t* residues);
+
 /* Host copy of the schedule: order[j] = caller index of the j-th sequence in
  * length-descending order (host int32 [nseq]). */
 hmg_status hmg_db_order(const hmg_db* db, int32_t* order);

@@ -923,6 +923,16 @@ int64_t hmg_db_nseq(const hmg_db* db) { return db ? db->nseq : -1; }
 int64_t hmg_db_residues(const hmg_db* db) { return db ? db->residues : -1; }
 int64_t hmg_db_packed_bytes(const hmg_db* db) { return db ? std::max<int64_t>(db->nwords, 4) * 4 : -1; }
 
+int64_t hmg_db_long_lane(const hmg_db* db, int64_t* residues) {
+  if (!db) return -1;
+  if (residues) {
+    int64_t r = 0;
+    for (int64_t j = 0; j < db->nlong; ++j) r += db->len_sorted[j];
+    *residues = r;
+  }
+  return db->nlong;
+}
+
 hmg_status hmg_db_order(const hmg_db* db, int32_t* order) {
   if (!db || (!order && db->nseq)) return HMG_EINVAL;
   std::copy(db->order.begin(), db->order.end(), order);

@@ -134,9 +134,8 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
     w4.x = w4.y;
     w4.y = w4.z;
     w4.z = w4.w;
-#pragma unroll
-    for (int j = 0; j < 6; ++j) {
-      const int x = (w >> (5 * j)) & 31;
+    // one DP row (Alg 1 l.11-20); `check`: per-row J->B / overflow vote
+    auto row = [&](int x, bool check) {
       uint32_t e[Q];
       load_row<G, Q>(sm + x * ROWW, z, e);
       // diagonal carry from the previous virtual lane (value after its emission)
@@ -149,6 +148,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
 #pragma unroll
       for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
       if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+      if (!check) return;
       // does any cell of this row reach the J->B / overflow threshold?
       const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
       const unsigned bal = __ballot_sync(0xffffffffu, hit);
@@ -172,6 +172,27 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
           }
         }
       }
+    };
+    if constexpr (Q <= 8) {
+      // short rows: vote once per word (6 rows).  R is a running max, so a threshold crossing
+      // anywhere in the word shows at its end; then the word is replayed from a snapshot
+      // with the per-row vote (exact, and rare: only hits).
+      uint32_t ts[Q];
+#pragma unroll
+      for (int q = 0; q < Q; ++q) ts[q] = t[q];
+      const uint32_t Rs = R;
+#pragma unroll
+      for (int j = 0; j < 6; ++j) row((w >> (5 * j)) & 31, false);
+      if (__any_sync(0xffffffffu, (__vadd2(R, thrv) & 0x80008000u) != 0u)) {
+#pragma unroll
+        for (int q = 0; q < Q; ++q) t[q] = ts[q];
+        R = Rs;
+#pragma unroll
+        for (int j = 0; j < 6; ++j) row((w >> (5 * j)) & 31, true);
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < 6; ++j) row((w >> (5 * j)) & 31, true);
     }
    }
   }

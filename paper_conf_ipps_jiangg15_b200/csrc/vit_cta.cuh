@@ -47,7 +47,7 @@ struct VitCtaSmem {
 };
 
 template <int W, int Q>
-__global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
+__global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const VitArgs a) {
   using S = VitCtaSmem<W, Q>;
   static_assert(Q % 2 == 0, "Q must be even (s16 emission pairs)");
   extern __shared__ uint4 smem4[];
@@ -64,13 +64,15 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
   const int w = g >> 5, lane = g & 31;
 
   // transitions of this thread's nodes (into-k BM MM IM DM, out-of-k MD MI II DD), s32
-  int tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
+  // (B->M_k is re-read from global memory: it only matters when xB changes)
+  int tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
   int ps[Q], wout[Q];
+  const int32_t* tBMg = a.tr + g * Q;
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     const int o = g * Q + q;
     const int NQ = S::NT * Q;
-    tBM[q] = a.tr[0 * NQ + o]; tMM[q] = a.tr[1 * NQ + o]; tIM[q] = a.tr[2 * NQ + o]; tDM[q] = a.tr[3 * NQ + o];
+    tMM[q] = a.tr[1 * NQ + o]; tIM[q] = a.tr[2 * NQ + o]; tDM[q] = a.tr[3 * NQ + o];
     tMD[q] = a.tr[4 * NQ + o]; tMI[q] = a.tr[5 * NQ + o]; tII[q] = a.tr[6 * NQ + o]; tDD[q] = a.tr[7 * NQ + o];
   }
   int bsum = 0;
@@ -131,7 +133,7 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       Mc[q] = Ic[q] = Dc[q] = kNegW;                                  // Alg 2 l.9
-      Bk[q] = sadd(kBaseW + move, tBM[q]);
+      Bk[q] = sadd(kBaseW + move, __ldg(tBMg + q));
     }
     int R = kNegW, xJ = kNegW;
     bool ovf = false;
@@ -241,7 +243,7 @@ __global__ void __launch_bounds__(32 * W) vit_cta_kernel(const VitArgs a) {
             xJ = m - 500;
             const int xB = max(xJ, kBaseW) + move;
 #pragma unroll
-            for (int q = 0; q < Q; ++q) Bk[q] = sadd(xB, tBM[q]);
+            for (int q = 0; q < Q; ++q) Bk[q] = sadd(xB, __ldg(tBMg + q));
             thr = min(max(xJ, kBaseW) + 501, 32767);
           }
         }

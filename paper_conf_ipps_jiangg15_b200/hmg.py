@@ -42,6 +42,7 @@ SIGNATURES = {
     "hmg_db_nseq": (c_i64, [c_p]),
     "hmg_db_residues": (c_i64, [c_p]),
     "hmg_db_packed_bytes": (c_i64, [c_p]),
+    "hmg_db_long_lane": (c_i64, [c_p, c_p]),
     "hmg_db_order": (c_int, [c_p, c_p]),
     "hmg_db_image": (c_int, [c_p, c_p]),
     "hmg_db_upload": (c_int, [c_p, c_p, c_p]),
@@ -182,6 +183,12 @@ class Database:
     @property
     def packed_bytes(self) -> int:
         return lib().hmg_db_packed_bytes(self._h)
+
+    def long_lane(self):
+        """(number of long-lane sequences, their residues) -- DESIGN.md 4.4."""
+        r = ctypes.c_int64()
+        n = lib().hmg_db_long_lane(self._h, ctypes.byref(r))
+        return int(n), int(r.value)
 
     def order(self) -> np.ndarray:
         o = np.zeros(self.nseq, dtype=np.int32)
