@@ -146,6 +146,7 @@ cudaError_t launch_vit_cta(int W, int Q, const VitArgs& a, cudaStream_t st, int*
 size_t vit_cta_smem(int W, int Q);
 int long_msv_q(int QV);
 int msv_q_max(int G);
+int msv_table_words(int G, int Q);   // MsvLayout<G, Q>::WORDS
 int vit_q_max(int G);
 
 // pipeline helpers (pipeline.cu)

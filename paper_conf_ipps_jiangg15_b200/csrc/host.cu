@@ -215,14 +215,22 @@ std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
     if (x >= kAlpha || node > M) return kNegE;
     return (int16_t)(p.bias - (int)p.cost[(size_t)x * M + (node - 1)]);
   };
-  for (int x = 0; x < kRows; ++x)
-    for (int z = 0; z < G; ++z)
-      for (int q = 0; q < Q; ++q) {
-        const uint16_t lo = (uint16_t)e_of(x, z * Q + q + 1);
-        const uint16_t hi = (uint16_t)e_of(x, (z + G) * Q + q + 1);
-        t[(size_t)x * ROWW + word_index(z, q)] = (uint32_t)lo | ((uint32_t)hi << 16);
-      }
-  return t;
+  // MsvLayout<G, Q> (msv.cuh): G < 8 -> 8/G copies, rows padded to 128 B, copy k shifted 16*G*k B
+  const int ncopy = G < 8 ? 8 / G : 1;
+  const int stride = ncopy > 1 ? (ROWW + 31) / 32 * 32 : ROWW;
+  const int copy = kRows * stride;
+  std::vector<uint32_t> out((size_t)msv_table_words(G, Q), 0u);
+  for (int k = 0; k < ncopy; ++k)
+    for (int x = 0; x < kRows; ++x)
+      for (int z = 0; z < G; ++z)
+        for (int q = 0; q < Q; ++q) {
+          const uint16_t lo = (uint16_t)e_of(x, z * Q + q + 1);
+          const uint16_t hi = (uint16_t)e_of(x, (z + G) * Q + q + 1);
+          out[(size_t)k * (copy + 4 * G) + (size_t)x * stride + word_index(z, q)] =
+              (uint32_t)lo | ((uint32_t)hi << 16);
+        }
+  (void)t;
+  return out;
 }
 
 // Viterbi register-kernel tables: emissions as s32 in the MSV chunk layout over Q words per lane
@@ -1115,7 +1123,12 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       int ok = 0;
       int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
       nb = env_int("HMG_PIPE_LONG_SMS", nb);
-      const bool sync_mode = env_int("HMG_LONG_SYNC", 0) != 0;   // diagnostics: no overlap
+      // Default: the long-lane Viterbi kernel waits for the chunked MSV through a stream event
+      // (it then needs no inter-kernel spinning, so serialised execution -- ncu, sanitizers,
+      // CUDA_LAUNCH_BLOCKING -- cannot deadlock); its side stream has the highest priority so its
+      // blocks are placed before the main MSV kernel's.  HMG_LONG_SPIN=1 instead launches it first
+      // and lets it wait per sequence on device flags (more overlap, not serialisation-safe).
+      const bool sync_mode = env_int("HMG_LONG_SPIN", 0) == 0;
       if (sync_mode) {
         if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
         if (!ok) return HMG_EUNSUPPORTED;

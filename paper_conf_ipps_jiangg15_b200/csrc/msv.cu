@@ -20,6 +20,16 @@ const void* msv_fast_ptr_g32(int q);
 
 int msv_q_max(int G) { return G == 32 ? 40 : 32; }
 
+int msv_table_words(int G, int Q) {
+  switch (G) {
+    case 4: {
+      const int stride = (Q * 4 + 31) / 32 * 32, copy = kRows * stride;
+      return ((2 * copy + 16) + 3) / 4 * 4;
+    }
+    default: return kRows * Q * G;
+  }
+}
+
 static const void* msv_fast_ptr(int G, int Q) {
   switch (G) {
     case 4: return msv_fast_ptr_g4(Q);
@@ -35,7 +45,7 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
   const int QL = (G == 32) ? 0 : (G * Q + 31) / 32;
-  const size_t smem = ((size_t)kRows * Q * G + (size_t)kRows * QL * 32) * 4;
+  const size_t smem = ((size_t)msv_table_words(G, Q) + (size_t)kRows * QL * 32) * 4;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = 0, per = 0;

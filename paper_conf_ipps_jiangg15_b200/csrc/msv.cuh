@@ -39,6 +39,19 @@ struct Chunks {
   static constexpr bool has1 = (r % 2) == 1;
 };
 
+// Shared-memory layout of the striped table for lane groups of G.  For G < 8 two or more
+// groups share a quarter-warp's LDS.128 wavefront while reading different residue rows; they
+// get their own copy of the table, shifted by 16*G bytes inside the 128-byte bank period
+// (row stride a multiple of 128 B), so their 16*G-byte chunks never share a bank.
+template <int G, int Q>
+struct MsvLayout {
+  static constexpr int NCOPY = G < 8 ? 8 / G : 1;
+  static constexpr int STRIDE = NCOPY > 1 ? (Q * G + 31) / 32 * 32 : Q * G;     // words per row
+  static constexpr int COPY = kRows * STRIDE;                                   // words per copy
+  static constexpr int WORDS = ((NCOPY * COPY + (NCOPY - 1) * 4 * G) + 3) / 4 * 4;
+  __host__ __device__ static constexpr int base(int grp) { return (grp % NCOPY) * (COPY + 4 * G); }
+};
+
 template <int G, int Q>
 __device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z, uint32_t (&e)[Q]) {
   using C = Chunks<Q>;
@@ -94,10 +107,12 @@ __device__ __forceinline__ int msv_thr(int xJ, int bias) {
 template <int G, int Q>
 __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
                                          long long send) {
-  constexpr int ROWW = Q * G;              // words per residue row
+  // sm: the table as laid out by MsvLayout<G, Q>
+  constexpr int ROWW = MsvLayout<G, Q>::STRIDE;    // words per residue row
   const int lane = threadIdx.x & 31;
   const int z = lane & (G - 1);
   const int grp = lane / G;
+  sm += MsvLayout<G, Q>::base(grp);
   const unsigned gbits = (G == 32 ? 0xffffffffu : ((1u << G) - 1u)) << (grp * G);
   const uint32_t sel = (z == 0) ? 0x1054u : 0x3210u;   // carry fix-up for virtual lane 0 / G
   const uint32_t negpair = (uint32_t)(uint16_t)kNegE;  // low half = -inf
@@ -279,7 +294,7 @@ template <int G, int Q>
 __global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
   extern __shared__ uint4 smem4[];
   constexpr int QL = MsvLong<G, Q>::QL;
-  constexpr int W0 = kRows * Q * G;        // words of the main table
+  constexpr int W0 = MsvLayout<G, Q>::WORDS;   // words of the main table (all copies)
   constexpr int W1 = kRows * QL * 32;      // words of the long-sequence table
   {
     const uint4* src = reinterpret_cast<const uint4*>(a.prof);
