@@ -58,8 +58,8 @@ struct VitArgs {
   int64_t ndone;
 };
 
-// Pipeline long lane (long.cu): chunked whole-warp MSV for the longest sequences, then
-// whole-warp Viterbi for their MSV survivors on SMs held alone, concurrent with the main MSV.
+// Long-sequence lane (long.cu): chunked whole-warp MSV for the longest sequences and, in the
+// pipeline, whole-warp Viterbi for their MSV survivors on SMs held alone.
 struct LongArgs {
   MsvArgs m;                 // m.prof = whole-warp MSV table (32, QL), m.raw = MSV raw (sorted)
   VitArgs v;                 // v.rsc / v.tr = register-kernel tables (32, QV), v.raw_sorted
@@ -71,7 +71,6 @@ struct LongArgs {
   int chunk_rows;
   int* chunk_max;            // [nitems]
   unsigned* chunk_done;      // [nlong] chunks finished
-  unsigned* ready;           // [nlong] 1 once the MSV raw / owned flag of the sequence are final
   unsigned long long* counter;  // [2] work queues (chunks, Viterbi)
 };
 
@@ -136,7 +135,7 @@ struct hmg_db {
 namespace hmg {
 extern std::atomic<long long> g_launches;   // kernels launched by libhmg (hmg_kernel_launches)
 // kernels / launchers (CUDA side)
-cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int* ok, bool pdl = false);
 cudaError_t launch_msv_exact(const MsvArgs& a, int nwarps, cudaStream_t st);
 cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
@@ -162,4 +161,5 @@ cudaError_t to_sorted_ids(const int32_t* caller_ids, int64_t n, const int32_t* i
                           cudaStream_t st);
 cudaError_t set_count(int64_t* d, int64_t v, cudaStream_t st);
 size_t scan_tmp_bytes(int64_t n);
+
 }  // namespace hmg

@@ -167,7 +167,7 @@ int env_int(const char* name, int dflt) {
 // ---------------------------------------------------------------- kernel geometry
 void msv_geometry(int M, int* G, int* Q) {
   // lane-group size from the G sweep on the config-2 DB (profiles/msv_sweep_r01.txt)
-  int g = M < 80 ? 8 : M < 150 ? 16 : M <= 450 ? 8 : M <= 640 ? 16 : 32;
+  int g = M < 80 ? 4 : M <= 450 ? 8 : M <= 640 ? 16 : 32;
   const int o = env_int("HMG_MSV_G", 0);
   if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
   // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
@@ -392,7 +392,8 @@ double mean_len(const hmg_db* db) { return db->nseq ? (double)db->residues / (do
 // MSV fast kernel over the DB into raw_sorted (device, sorted order).  pipe_nlong >= 0: the
 // first pipe_nlong sequences are scored by the pipeline long lane instead.
 hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S,
-                        int64_t pipe_nlong) {
+                        int64_t pipe_nlong, bool pdl = false, bool mark0 = true,
+                        unsigned long long* ctr_zeroed = nullptr) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
@@ -404,15 +405,20 @@ hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st,
     a.nlong = count_longer(db, env_int("HMG_MSV_LLONG", (int)std::max(1000.0, 8.0 * mean_len(db))));
     a.skip_long = 0;
   }
-  auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
-  if (e) return cuda_status(e);
-  if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+  // (with pdl the counters must be zeroed before the preceding kernel: any stream operation
+  //  between it and this launch would serialise them)
+  auto* ctr = ctr_zeroed;
+  if (!ctr) {
+    ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+    if (e) return cuda_status(e);
+    if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+  }
   a.counter = ctr;
   const int nwarps_exact = 148 * 16;
   if (p->msv_fast && p->msv_Q > 0) {
     int ok = 0;
-    mark(0, st);
-    if ((e = launch_msv_fast(p->msv_G, p->msv_Q, a, st, &ok))) return cuda_status(e);
+    if (mark0) mark(0, st);
+    if ((e = launch_msv_fast(p->msv_G, p->msv_Q, a, st, &ok, pdl))) return cuda_status(e);
     if (!ok) return HMG_EUNSUPPORTED;
     mark(1, st);
   } else {
@@ -457,13 +463,14 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
 // the lane-group kernel; then the exact re-score of flagged sequences.
 hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
   int64_t nlong = -1;
+  mark(0, st);
   if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && db->nlong > 0 && !env_int("HMG_NO_LONG_LANE", 0)) {
     LongArgs la{};
     hmg_status s = run_msv_long_chunks(p, db, st, raw_sorted, S, &la);
     if (s != HMG_OK) return s;
     nlong = db->nlong;
   }
-  hmg_status s = run_msv_fast(p, db, st, raw_sorted, S, nlong);
+  hmg_status s = run_msv_fast(p, db, st, raw_sorted, S, nlong, false, false);
   if (s != HMG_OK) return s;
   return run_msv_redo(p, db, st, raw_sorted, S);
 }
@@ -476,10 +483,10 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
   auto* owned = (uint8_t*)S.get((size_t)nlong, &e);
   auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
   auto* cmax = (int*)S.get(sizeof(int) * (size_t)std::max<int64_t>(db->nchunks, 1), &e);
-  auto* cdone = (unsigned*)S.get(sizeof(unsigned) * 2 * (size_t)nlong, &e);   // chunk_done | ready
+  auto* cdone = (unsigned*)S.get(sizeof(unsigned) * (size_t)nlong, &e);
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
-  if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * 2 * (size_t)nlong, st))) return cuda_status(e);
+  if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * (size_t)nlong, st))) return cuda_status(e);
   LongArgs& la = *la_out;
   la = LongArgs{};
   la.m = msv_args(p, db);
@@ -492,41 +499,16 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
   la.chunk_rows = db->chunk_rows;
   la.chunk_max = cmax;
   la.chunk_done = cdone;
-  la.ready = cdone + nlong;
   la.counter = lctr;
   int ok = 0;
   if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
   return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 
-// per-device side stream + fork/join events for the pipeline long lane
-struct SideStream {
-  cudaStream_t s = nullptr;
-  cudaEvent_t fork = nullptr, join = nullptr;
-};
-SideStream g_side[64];
-std::mutex g_side_mu;
-
-hmg_status side_stream(int dev, SideStream** out) {
-  if (dev < 0 || dev >= 64) return HMG_EINVAL;
-  std::lock_guard<std::mutex> g(g_side_mu);
-  SideStream& S = g_side[dev];
-  if (!S.s) {
-    int lo = 0, hi = 0;
-    cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    cudaError_t e = cudaStreamCreateWithPriority(&S.s, cudaStreamNonBlocking, hi);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&S.fork, cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&S.join, cudaEventDisableTiming);
-    if (e != cudaSuccess) return cuda_status(e);
-  }
-  *out = &S;
-  return HMG_OK;
-}
-
 // Viterbi over sorted-order ids (list, device count) into raw_sorted.
 hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
                    cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr,
-                   int64_t ndone = 0) {
+                   int64_t ndone = 0, bool marks = true) {
   cudaError_t e = cudaSuccess;
   VitArgs a{};
   a.words = db->d_words;
@@ -546,7 +528,7 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
   a.counter = ctr;
-  mark(3, st);
+  if (marks) mark(3, st);
   if (!p->vit_generic && p->vit_W > 0) {
     int ok = 0;
     if ((e = launch_vit_cta(p->vit_W, p->vit_Q, a, st, &ok))) return cuda_status(e);
@@ -562,7 +544,7 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     a.scratch = scr;
     if ((e = launch_vit_generic(a, nwarps, st))) return cuda_status(e);
   }
-  mark(4, st);
+  if (marks) mark(4, st);
   return HMG_OK;
 }
 
@@ -1079,25 +1061,20 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     void* tmp = S.get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
     if (e) return cuda_status(e);
     mark_reset();
-    // pipeline long lane (long.cu): chunked whole-warp MSV of the longest sequences, then their
-    // Viterbi on SMs held alone (side stream) while the main MSV kernel runs on the others
+    // pipeline long lane (long.cu): chunked MSV of the longest sequences on the whole GPU, then
+    // their Viterbi filter on SMs held alone by pipe_long_vit_kernel while the main MSV kernel
+    // (programmatic dependent launch) fills the other SMs
     const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && !p->vit_generic && p->vit_W == 0 &&
                            !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
-    SideStream* side = nullptr;
+    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+    if (e) return cuda_status(e);
+    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+    mark(0, st);
     if (nlong > 0) {
-      if ((s = side_stream(db->device, &side)) != HMG_OK) return s;
-      owned = (uint8_t*)S.get((size_t)nlong, &e);
-      auto* lctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
-      auto* cmax = (int*)S.get(sizeof(int) * (size_t)std::max<int64_t>(db->nchunks, 1), &e);
-      auto* cdone = (unsigned*)S.get(sizeof(unsigned) * 2 * (size_t)nlong, &e);   // chunk_done | ready
-      if (e) return cuda_status(e);
-      if ((e = cudaMemsetAsync(lctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
-      if ((e = cudaMemsetAsync(cdone, 0, sizeof(unsigned) * 2 * (size_t)nlong, st))) return cuda_status(e);
       LongArgs la{};
-      la.m = msv_args(p, db);
-      la.m.prof = p->d_long_msv;
-      la.m.raw = raw_sorted;
+      if ((s = run_msv_long_chunks(p, db, st, raw_sorted, S, &la)) != HMG_OK) return s;
+      owned = la.owned;
       la.v.words = db->d_words;
       la.v.woff16 = db->d_woff16;
       la.v.len = db->d_len;
@@ -1108,42 +1085,14 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       la.v.M = p->M;
       la.v.raw_sorted = vraw_sorted;
       la.thr = tm;
-      la.owned = owned;
-      la.nlong = nlong;
-      la.chunk_start = db->d_chunk_start;
-      la.nitems = db->nchunks;
-      la.chunk_rows = db->chunk_rows;
-      la.chunk_max = cmax;
-      la.chunk_done = cdone;
-      la.ready = cdone + nlong;
-      la.counter = lctr;
-      // Viterbi of the long survivors on a side stream, on SMs held alone.  It is enqueued
-      // first so its blocks are placed before the main MSV kernel fills the GPU, and it waits
-      // per sequence (ready[]) for the chunked MSV below, which runs on the other SMs.
-      int ok = 0;
+      // blocks (SMs) for the long-survivor Viterbi: about one per 20 long sequences, 2..16
       int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
       nb = env_int("HMG_PIPE_LONG_SMS", nb);
-      // Default: the long-lane Viterbi kernel waits for the chunked MSV through a stream event
-      // (it then needs no inter-kernel spinning, so serialised execution -- ncu, sanitizers,
-      // CUDA_LAUNCH_BLOCKING -- cannot deadlock); its side stream has the highest priority so its
-      // blocks are placed before the main MSV kernel's.  HMG_LONG_SPIN=1 instead launches it first
-      // and lets it wait per sequence on device flags (more overlap, not serialisation-safe).
-      const bool sync_mode = env_int("HMG_LONG_SPIN", 0) == 0;
-      if (sync_mode) {
-        if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
-        if (!ok) return HMG_EUNSUPPORTED;
-      }
-      if ((e = cudaEventRecord(side->fork, st))) return cuda_status(e);
-      if ((e = cudaStreamWaitEvent(side->s, side->fork, 0))) return cuda_status(e);
-      if ((e = launch_pipe_long_vit(p->long_QV, la, nb, side->s, &ok))) return cuda_status(e);
+      int ok = 0;
+      if ((e = launch_pipe_long_vit(p->long_QV, la, nb, st, &ok))) return cuda_status(e);
       if (!ok) return HMG_EUNSUPPORTED;
-      if ((e = cudaEventRecord(side->join, side->s))) return cuda_status(e);
-      if (!sync_mode) {
-        if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);   // main stream
-        if (!ok) return HMG_EUNSUPPORTED;
-      }
     }
-    s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1);     // Fig 1: MSV
+    s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV
     if (s != HMG_OK) return s;
     s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;
@@ -1152,7 +1101,7 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     if (e) return cuda_status(e);
     s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S, owned, nlong);  // P7Viterbi on survivors
     if (s != HMG_OK) return s;
-    if (nlong > 0 && (e = cudaStreamWaitEvent(st, side->join, 0))) return cuda_status(e);
+
     e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st);
     mark(5, st);
   }

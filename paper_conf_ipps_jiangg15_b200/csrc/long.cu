@@ -1,20 +1,22 @@
-// long.cu -- the pipeline's long lane: the longest sequences (L > ~8x the mean length).
+// long.cu -- the long-sequence lane (sequences with L > ~8x the mean length).
 //
 // A DP row cannot be split across time (Alg 1/2 carry xB from row i to i+1), so a
 // sequence's filter time is bounded below by its length times the row latency of one
 // lane group; and the B200 warp arbiter shares issue slots evenly among resident warps
 // (measured, profiles/arbiter_r01.txt), so a long sequence sharing its SM sub-partition
-// with five other warps runs five to six times slower than alone.  Two kernels:
+// with five other warps runs five to six times slower than alone.
 //
-// pipe_long_msv_kernel<QL>: MSV of the long sequences cut into row chunks that run in
-//   parallel, each from the empty state M rows early (exact: an MSV domain is one ungapped
-//   diagonal, so row i depends only on rows > i - M while xB is unchanged).  The last
-//   chunk of a sequence to finish combines the chunk maxima; if any chunk saw a row that
-//   could move xB (a hit) or overflow, it re-runs the sequence with the sequential
-//   whole-warp DP (msv_batch<32, QL>).  It runs on the main stream before the main MSV.
-// pipe_long_vit_kernel<QV>: Viterbi filter (whole warp, latency variant of VitLane) of the
-//   long MSV survivors, longest first, on SMs it holds alone (each block asks for most of
-//   the shared memory), concurrently with the main MSV kernel on the other SMs.
+// MSV of a long sequence is cut into row chunks that run in parallel, each from the empty
+// state M rows early.  Exact while xB is unchanged: an MSV domain is one ungapped diagonal,
+// so row i depends only on rows > i - M.  The last chunk of a sequence to finish combines
+// the chunk maxima; if any chunk saw a row that could move xB (a hit) or overflow, it
+// re-runs the sequence with the sequential whole-warp DP (msv_batch<32, QL>).
+//   pipe_long_msv_kernel<QL>   chunked MSV only (hmg_msv), on the whole GPU before the main
+//                              MSV kernel;
+//   pipe_long_vit_kernel<QV>   the Viterbi filter (latency variant of VitLane) of the long
+//                              sequences that pass, on SMs it holds alone, while the main MSV
+//                              kernel (programmatic dependent launch) fills the other SMs
+//                              (hmg_pipeline).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -87,17 +89,23 @@ __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
     } else {
       raw = msv_batch<32, QL>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
     }
-    if (lane == 0) {
-      A.owned[j] = raw != 254;                  // 254: exact re-score on the main stream decides
-      __threadfence();
-      atomicExch(A.ready + j, 1u);              // publish to pipe_long_vit_kernel
-    }
+    if (lane == 0) A.owned[j] = raw != 254;
   }
 }
 
+
+// Viterbi filter of the long sequences that passed MSV (pipeline only): one warp per sequence,
+// longest first, on blocks that each ask for most of an SM's shared memory (so they hold their
+// SMs alone).  Every block executes griddepcontrol.launch_dependents as soon as it is resident;
+// the main MSV kernel is launched next in the same stream with programmatic stream
+// serialisation, so it is dispatched only after these blocks are placed and then fills the
+// other SMs while this kernel runs.  Its inputs (raw MSV scores of the long sequences) come
+// from pipe_long_msv_kernel, which completed before it in stream order: nothing waits on a
+// concurrently running kernel, so serialised execution (profilers, sanitizers) stays correct.
 template <int QV>
 __global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
-  constexpr int WV = kRows * QV * 32;        // Viterbi emission table words
+  asm volatile("griddepcontrol.launch_dependents;");
+  constexpr int WV = kRows * QV * 32;
   extern __shared__ uint4 smem4[];
   {
     const uint4* s1 = reinterpret_cast<const uint4*>(A.v.rsc);
@@ -113,23 +121,15 @@ __global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
     if (lane == 0) b = atomicAdd(A.counter + 1, 1ull);
     b = __shfl_sync(0xffffffffu, b, 0);
     if ((long long)b >= A.nlong) break;
-    const int s = (int)b;
-    // wait until the MSV of sequence s is final (pipe_long_msv_kernel runs concurrently on the
-    // other SMs and finishes the longest sequences first)
-    if (lane == 0) {
-      while (atomicAdd(A.ready + s, 0u) == 0u) __nanosleep(256);
-      __threadfence();
-    }
-    __syncwarp();
-    if (!*((volatile uint8_t*)A.owned + s)) continue;
-    const int raw = *((volatile uint8_t*)A.m.raw + s);
-    const int L = A.m.len[s];
+    const int j = (int)b;
+    if (!A.owned[j]) continue;                   // 254: the exact re-score + main stage decide
+    const int raw = A.m.raw[j];
+    const int L = A.m.len[j];
     if (!(raw == 255 || raw >= (int)A.thr[L])) continue;       // MSV pass flag (reading R25)
-    const uint32_t* wp = A.v.words + (size_t)A.v.woff16[s] * 4;
-    const int nw = (L + 5) / 6;
+    const uint32_t* wp = A.v.words + (size_t)A.v.woff16[j] * 4;
     V.start(A.v.move[L], true);
     ResStream rs;
-    rs.init(wp, nw);
+    rs.init(wp, (L + 5) / 6);
     for (int iq = 0; iq < rs.nq; ++iq) {                        // Alg 2 row loop
       uint4 w4 = rs.next(iq);
 #pragma unroll 1
@@ -139,14 +139,14 @@ __global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
         w4.y = w4.z;
         w4.z = w4.w;
 #pragma unroll
-        for (int j = 0; j < 6; ++j) {
-          const int x = (w >> (5 * j)) & 31;
+        for (int jj = 0; jj < 6; ++jj) {
+          const int x = (w >> (5 * jj)) & 31;
           V.row(smv + x * (QV * 32), lane, 0xffffffffu);
         }
       }
     }
     const int vraw = V.finish();
-    if (lane == 0) A.v.raw_sorted[s] = (int16_t)vraw;
+    if (lane == 0) A.v.raw_sorted[j] = (int16_t)vraw;
   }
 }
 
@@ -191,32 +191,22 @@ cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int
   return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args, smem, st);
 }
 
+}  // namespace hmg
+
+namespace hmg {
 cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
   const void* fn = pick_vit<1>(QV);
-  const void* producer = pick_msv<1>(long_msv_q_of(QV));
-  *ok = fn != nullptr && producer != nullptr;
-  if (!*ok) return cudaSuccess;
-  // This kernel spins on flags the chunked-MSV kernel sets.  With CUDA's lazy module loading the
-  // first launch of a kernel may synchronise the context, which would wait on this spinning
-  // kernel forever: force both kernels to be loaded before this one is launched.
-  cudaFuncAttributes fa;
-  cudaError_t e0 = cudaFuncGetAttributes(&fa, producer);
-  if (e0 == cudaSuccess) e0 = cudaFuncGetAttributes(&fa, fn);
-  if (e0 != cudaSuccess) return e0;
-  // ask for most of the SM's shared memory so no block of another kernel shares the SM
+  *ok = fn != nullptr;
+  if (!fn) return cudaSuccess;
   const size_t need = (size_t)kRows * QV * 32 * 4;
   int dev = 0, maxsm = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-  const size_t smem = std::max(need, (size_t)maxsm - 8192);
+  const size_t smem = std::max(need, (size_t)maxsm - 8192);   // hold the SM alone
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  const size_t psmem = (size_t)kRows * long_msv_q_of(QV) * 32 * 4;
-  e = cudaFuncSetAttribute(producer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem);
   if (e != cudaSuccess) return e;
   void* args[] = {const_cast<LongArgs*>(&a)};
   g_launches += 1;
   return cudaLaunchKernel(fn, dim3((unsigned)nblocks), dim3(128), args, smem, st);
 }
-
 }  // namespace hmg

@@ -40,7 +40,7 @@ static const void* msv_fast_ptr(int G, int Q) {
   return nullptr;
 }
 
-cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int* ok) {
+cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int* ok, bool pdl) {
   const void* fn = msv_fast_ptr(G, Q);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
@@ -60,7 +60,20 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
   if (grid < 1) grid = 1;
   void* args[] = {const_cast<MsvArgs*>(&a)};
   g_launches += 1;
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args, smem, st);
+  if (!pdl) return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args, smem, st);
+  // programmatic dependent launch: may start once every block of the preceding kernel in the
+  // stream (the pipeline long lane) is resident and has signalled griddepcontrol.launch_dependents
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelExC(&cfg, fn, args);
 }
 
 __device__ __forceinline__ int u8sat(int v) { return v < 0 ? 0 : (v > 255 ? 255 : v); }

@@ -351,13 +351,14 @@ def test_vit_block_kernel_delete_chains(M, monkeypatch):
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
 
 
-@pytest.mark.parametrize("chunk,spin", [(1032, "0"), (60, "0"), (1032, "1")])
-def test_pipeline_long_lane(chunk, spin, monkeypatch):
+@pytest.mark.parametrize("chunk,sms", [(1032, "0"), (60, "0"), (1032, "2")])
+def test_pipeline_long_lane(chunk, sms, monkeypatch):
     """The pipeline long lane: sequences longer than max(1500, 8 x mean) get chunked MSV (rows
     from the empty state M rows early) and whole-warp Viterbi on a side stream.  Strong planted
     hits in some long sequences force the sequential fallback (a chunk sees a J->B row)."""
     monkeypatch.setenv("HMG_PIPE_CHUNK", str(chunk))
-    monkeypatch.setenv("HMG_LONG_SPIN", spin)
+    if sms != "0":
+        monkeypatch.setenv("HMG_PIPE_LONG_SMS", sms)
     rng = np.random.default_rng(42)
     prof = synth.make_profile(120, 4242)
     best = np.argmax(prof.msc[:, :20], axis=1).astype(np.uint8)
