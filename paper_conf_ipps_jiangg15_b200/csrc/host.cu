@@ -14,6 +14,7 @@
 #include <cstring>
 #include <new>
 #include <numeric>
+#include <random>
 #include <vector>
 
 #include "hmg_internal.h"
@@ -757,6 +758,86 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     return st;
   }
   *out = p;
+  return HMG_OK;
+}
+
+hmg_status hmg_profile_set_ev(hmg_profile* p, const hmg_evparams* ev) {
+  if (!p || !ev || !(ev->lambda_msv > 0) || !(ev->lambda_vit > 0) || std::isnan(ev->mu_msv) ||
+      std::isnan(ev->mu_vit))
+    return HMG_EINVAL;
+  std::lock_guard<std::mutex> g(p->mu);
+  p->ev = *ev;
+  p->has_ev = true;
+  if (p->device >= 0) {
+    Dev dg(p->device);
+    cudaFree(p->thr_msv.d);
+    cudaFree(p->thr_vit.d);
+  }
+  p->thr_msv = hmg_profile::Thr();
+  p->thr_vit = hmg_profile::Thr();
+  return HMG_OK;
+}
+
+hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, double lambda, hmg_evparams* out) {
+  if (!p || !out || n < 1 || L < 1 || !(lambda > 0) || !p->has_tsc || p->device < 0) return HMG_EINVAL;
+  // HMMER3 amino background (reading R34) and 0.05% X, as the synthetic databases
+  static const double f[20] = {0.0787945, 0.0151600, 0.0535222, 0.0668298, 0.0397062, 0.0695071, 0.0229198,
+                               0.0590092, 0.0594422, 0.0963728, 0.0237718, 0.0414386, 0.0482904, 0.0395639,
+                               0.0540978, 0.0683364, 0.0540687, 0.0673417, 0.0114135, 0.0304133};
+  std::vector<double> w(f, f + 20);
+  double tot = 0;
+  for (double v : w) tot += v;
+  for (double& v : w) v = v / tot * (1.0 - 0.0005);
+  w.push_back(0.0005);
+  std::mt19937_64 rng(seed);
+  std::discrete_distribution<int> pick(w.begin(), w.end());
+  std::vector<uint8_t> dsq((size_t)n * L);
+  for (auto& c : dsq) {
+    const int k = pick(rng);
+    c = (uint8_t)(k == 20 ? 26 : k);
+  }
+  std::vector<int64_t> off((size_t)n + 1);
+  for (int i = 0; i <= n; ++i) off[i] = (int64_t)i * L;
+  hmg_db* db = nullptr;
+  hmg_status s = hmg_db_create(dsq.data(), off.data(), n, p->device, &db);
+  if (s != HMG_OK) return s;
+  Dev dg(p->device);
+  uint8_t* d_m = nullptr;
+  int16_t* d_v = nullptr;
+  cudaError_t e = cudaMalloc(&d_m, (size_t)n);
+  if (e == cudaSuccess) e = cudaMalloc(&d_v, sizeof(int16_t) * (size_t)n);
+  if (e == cudaSuccess) {
+    s = hmg_msv(p, db, 0.02, nullptr, d_m, nullptr);
+    if (s == HMG_OK) s = hmg_viterbi(p, db, nullptr, 0, 1e-3, nullptr, d_v, nullptr);
+  } else {
+    s = cuda_status(e);
+  }
+  std::vector<uint8_t> hm((size_t)n);
+  std::vector<int16_t> hv((size_t)n);
+  if (s == HMG_OK) {
+    e = cudaMemcpy(hm.data(), d_m, (size_t)n, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(hv.data(), d_v, sizeof(int16_t) * (size_t)n, cudaMemcpyDeviceToHost);
+    s = cuda_status(e);
+  }
+  cudaFree(d_m);
+  cudaFree(d_v);
+  hmg_db_destroy(db);
+  if (s != HMG_OK) return s;
+  const float null = null1_of(L);
+  auto fit = [&](auto nats_of, const auto& raw) {
+    double acc = 0;
+    int cnt = 0;
+    for (auto r : raw) {
+      const float nats = nats_of((int)r, L);
+      if (!std::isfinite(nats)) continue;
+      acc += exp(-lambda * ((double)(nats - null) / kLn2));
+      ++cnt;
+    }
+    return cnt ? -log(acc / cnt) / lambda : 0.0;
+  };
+  out->mu_msv = fit(msv_nats_of, hm);
+  out->mu_vit = fit(vit_nats_of, hv);
+  out->lambda_msv = out->lambda_vit = lambda;
   return HMG_OK;
 }
 

@@ -7,8 +7,7 @@
 //
 //   D->D (Lazy-F, Fig 7) is resolved as a max-plus carry chain.  Each thread's
 //   block of nodes maps an incoming D carry c to an outgoing max(cl, c + bsum), where cl is
-//   the outgoing carry computed directly from its M cells (max_q M_q + tMD_q + later tDD) and
-//   bsum the sum of its tDD.  Inside a warp the incoming carries are found by shuffles
+//   the outgoing carry of its in-thread D chain (carry-in -inf) and bsum the sum of its tDD.  Inside a warp the incoming carries are found by shuffles
 //   repeated while __any_sync reports a change (reading R19); across warps each warp
 //   publishes its outgoing carry, and after the barrier every warp folds the carries of the
 //   warps to its left itself (W <= 16 steps), so no further barrier round is needed.  With
@@ -66,7 +65,7 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
   // transitions of this thread's nodes (into-k BM MM IM DM, out-of-k MD MI II DD), s32
   // (B->M_k is re-read from global memory: it only matters when xB changes)
   int tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];
-  int ps[Q], wout[Q];
+  int ps[Q];
   const int32_t* tBMg = a.tr + g * Q;
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
@@ -80,14 +79,6 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
   for (int q = 0; q < Q; ++q) {
     ps[q] = bsum;                            // sum of tDD before node q inside the thread
     bsum += tDD[q];
-  }
-  {
-    int acc = 0;
-#pragma unroll
-    for (int q = Q - 1; q >= 0; --q) {
-      wout[q] = tMD[q] + acc;                // M_q -> D_{q+1} -> ... -> next thread's first node
-      acc += tDD[q];
-    }
   }
   // exclusive prefix of bsum over the lanes of the warp (constant), and warp totals
   int pbs = bsum;
@@ -157,8 +148,9 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
       int r[Q];
 #pragma unroll
       for (int h = 0; h < S::Q2; ++h) {
-        r[2 * h] = (int)(int16_t)(e2[h] & 0xffffu);
-        r[2 * h + 1] = (int)e2[h] >> 16;
+        // s16 -> s32 on the FMA pipe (IMAD.HI), which this ALU-bound kernel leaves idle
+        r[2 * h] = __mulhi((int)(e2[h] << 16), 65536);
+        r[2 * h + 1] = __mulhi((int)e2[h], 65536);
       }
       // diagonal carries (row i-1 at node g*Q): lane l-1, or lane 31 of warp w-1 (nb*)
       int cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
@@ -183,13 +175,11 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
       }
 #pragma unroll
       for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s32(R, Mc[q], Mc[q + 1]);
-      // D partial (l.17) + in-thread chain, and this thread's outgoing carry from its M cells
-      int cl = kNegW;
-#pragma unroll
-      for (int q = 0; q < Q; ++q) cl = __viaddmax_s32(Mc[q], wout[q], cl);
+      // D partial (l.17) + in-thread chain; this thread's outgoing carry is the chain's next link
       Dc[0] = kNegW;
 #pragma unroll
       for (int q = 1; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], sadd(Mc[q - 1], tMD[q - 1]));
+      const int cl = __viaddmax_s32(Dc[Q - 1], tDD[Q - 1], sadd(Mc[Q - 1], tMD[Q - 1]));
       // carries inside the warp: ci = outgoing of lane-1, iterate while any lane changes
       int out = cl, ci;
       for (;;) {
@@ -217,8 +207,25 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
       const int cw = w > 0 ? max(kNegW, pb_w + m1) : kNegW;
       const int cwl = w > 1 ? max(kNegW, pb_wl + m2) : kNegW;
       const int cf = max(ci, __viaddmax_s32(cw, pbs, kNegW));    // final carry into this thread
+      // apply the carry: D_q = max(D_q, cf + sum of the earlier tDD); runs die within a few
+      // nodes, so walk two and finish only if some thread still improves
+      {
+        bool imp = cf > Dc[0];
+        Dc[0] = max(Dc[0], cf);
+        constexpr int K0 = Q <= 4 ? Q : 2;
 #pragma unroll
-      for (int q = 0; q < Q; ++q) Dc[q] = __viaddmax_s32(cf, ps[q], Dc[q]);
+        for (int q = 1; q < K0; ++q) {
+          const int nd = __viaddmax_s32(Dc[q - 1], tDD[q - 1], kNegW);
+          imp = imp && nd > Dc[q];
+          Dc[q] = max(Dc[q], nd);
+        }
+        if constexpr (K0 < Q) {
+          if (__any_sync(0xffffffffu, imp)) {
+#pragma unroll
+            for (int q = K0; q < Q; ++q) Dc[q] = __viaddmax_s32(Dc[q - 1], tDD[q - 1], Dc[q]);
+          }
+        }
+      }
       // next row's diagonal carry for lane 0: warp w-1's last node, rebuilt here
       if (w > 0 && lane == 0) {
         const int* xc = scr + S::XC + (par * W + w - 1) * 4;

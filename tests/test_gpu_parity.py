@@ -240,6 +240,39 @@ def _calibrate(prof):
     return (oracle.fit_mu(np.array(mb), lam), lam, oracle.fit_mu(np.array(vb), lam), lam)
 
 
+@pytest.mark.parametrize("M", [64, 200, 700])
+def test_calibrate_matches_oracle_fit(M):
+    """hmg_calibrate (library RNG, GPU scoring) vs the oracle's fit on other background
+    sequences: the ML location for known lambda has SD ~ 1/(lambda sqrt(n)) = 0.046 bits at
+    n = 1000, so two independent fits agree within 0.3 bits (> 4.5 SD of the difference)."""
+    prof = synth.make_profile(M, 100 + M)
+    p = hmg.Profile(prof.msc, prof.tsc)
+    mu_m, lam_m, mu_v, lam_v = p.calibrate(n=1000, L=200, seed=11)
+    want = _calibrate(prof)
+    assert lam_m == lam_v == pytest.approx(math.log(2))
+    assert abs(mu_m - want[0]) < 0.3 and abs(mu_v - want[2]) < 0.3
+    # deterministic in the seed
+    assert p.calibrate(n=1000, L=200, seed=11) == (mu_m, lam_m, mu_v, lam_v)
+
+
+def test_profile_set_ev_rebuilds_thresholds():
+    """Pipeline flags after hmg_profile_set_ev equal those of a profile created with that ev."""
+    prof, db_ = synth.config(1)
+    dsq, off = db_.materialize()
+    ev = _calibrate(prof)
+    db = hmg.Database(dsq, off)
+    a = hmg.Profile(prof.msc, prof.tsc, ev=(ev[0] + 3, ev[1], ev[2] + 3, ev[3]))
+    oa = hmg.alloc_outputs(db.nseq)
+    hmg.hmg_pipeline(a, db, F1=0.05, F2=0.01, **oa)        # builds tables for the old ev
+    a.set_ev(ev)
+    hmg.hmg_pipeline(a, db, F1=0.05, F2=0.01, **oa)
+    b = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    ob = hmg.alloc_outputs(db.nseq)
+    hmg.hmg_pipeline(b, db, F1=0.05, F2=0.01, **ob)
+    torch.cuda.synchronize()
+    assert torch.equal(oa["flags"], ob["flags"]) and int(oa["n_survivors"]) == int(ob["n_survivors"])
+
+
 def _check_pipeline(prof, dsq, off, F1, F2, sample=None):
     ev = _calibrate(prof)
     p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
