@@ -104,12 +104,10 @@ void hmg_profile_destroy(hmg_profile* p);
  * seeded background sequences of length L (HMMER3 amino background, 0.05% X) that the library
  * scores on the profile's device with its own kernels: mu = -ln(mean(exp(-lambda * bits)))/lambda,
  * the closed-form ML location for known lambda.  Fills out (mu_*, lambda_* = lambda).
- * Needs a device profile with tsc; n >= 1, L >= 1, lambda > 0.  Synchronous. */
+ * Needs a device profile with tsc; n >= 1, L >= 1, lambda > 0.  Synchronous.  Profiles are
+ * immutable: create the searching profile with the returned parameters. */
 hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, double lambda, hmg_evparams* out);
 
-/* Replace the profile's Gumbel parameters (drops its cached threshold tables).  Not to be
- * called while compute calls using p are in flight. */
-hmg_status hmg_profile_set_ev(hmg_profile* p, const hmg_evparams* ev);
 
 /* ---------------------------------------------------------------- database */
 

@@ -761,23 +761,6 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   return HMG_OK;
 }
 
-hmg_status hmg_profile_set_ev(hmg_profile* p, const hmg_evparams* ev) {
-  if (!p || !ev || !(ev->lambda_msv > 0) || !(ev->lambda_vit > 0) || std::isnan(ev->mu_msv) ||
-      std::isnan(ev->mu_vit))
-    return HMG_EINVAL;
-  std::lock_guard<std::mutex> g(p->mu);
-  p->ev = *ev;
-  p->has_ev = true;
-  if (p->device >= 0) {
-    Dev dg(p->device);
-    cudaFree(p->thr_msv.d);
-    cudaFree(p->thr_vit.d);
-  }
-  p->thr_msv = hmg_profile::Thr();
-  p->thr_vit = hmg_profile::Thr();
-  return HMG_OK;
-}
-
 hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, double lambda, hmg_evparams* out) {
   if (!p || !out || n < 1 || L < 1 || !(lambda > 0) || !p->has_tsc || p->device < 0) return HMG_EINVAL;
   // HMMER3 amino background (reading R34) and 0.05% X, as the synthetic databases

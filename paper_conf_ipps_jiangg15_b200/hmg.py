@@ -57,7 +57,6 @@ SIGNATURES = {
     "hmg_strerror": (ctypes.c_char_p, [c_int]),
     "hmg_kernel_launches": (c_i64, []),
     "hmg_calibrate": (c_int, [c_p, c_int, c_int, ctypes.c_uint64, c_d, c_p]),
-    "hmg_profile_set_ev": (c_int, [c_p, c_p]),
     "hmg_set_stage_timing": (c_int, [c_int]),
     "hmg_stage_times": (c_int, [c_p]),
 }
@@ -155,10 +154,6 @@ class Profile:
         ev = hmg_evparams()
         _check(lib().hmg_calibrate(self._h, n, L, seed, lam, ctypes.byref(ev)), "hmg_calibrate")
         return (ev.mu_msv, ev.lambda_msv, ev.mu_vit, ev.lambda_vit)
-
-    def set_ev(self, ev):
-        e = hmg_evparams(*[float(v) for v in ev])
-        _check(lib().hmg_profile_set_ev(self._h, ctypes.byref(e)), "hmg_profile_set_ev")
 
     def close(self):
         if getattr(self, "_h", None):

@@ -255,24 +255,6 @@ def test_calibrate_matches_oracle_fit(M):
     assert p.calibrate(n=1000, L=200, seed=11) == (mu_m, lam_m, mu_v, lam_v)
 
 
-def test_profile_set_ev_rebuilds_thresholds():
-    """Pipeline flags after hmg_profile_set_ev equal those of a profile created with that ev."""
-    prof, db_ = synth.config(1)
-    dsq, off = db_.materialize()
-    ev = _calibrate(prof)
-    db = hmg.Database(dsq, off)
-    a = hmg.Profile(prof.msc, prof.tsc, ev=(ev[0] + 3, ev[1], ev[2] + 3, ev[3]))
-    oa = hmg.alloc_outputs(db.nseq)
-    hmg.hmg_pipeline(a, db, F1=0.05, F2=0.01, **oa)        # builds tables for the old ev
-    a.set_ev(ev)
-    hmg.hmg_pipeline(a, db, F1=0.05, F2=0.01, **oa)
-    b = hmg.Profile(prof.msc, prof.tsc, ev=ev)
-    ob = hmg.alloc_outputs(db.nseq)
-    hmg.hmg_pipeline(b, db, F1=0.05, F2=0.01, **ob)
-    torch.cuda.synchronize()
-    assert torch.equal(oa["flags"], ob["flags"]) and int(oa["n_survivors"]) == int(ob["n_survivors"])
-
-
 def _check_pipeline(prof, dsq, off, F1, F2, sample=None):
     ev = _calibrate(prof)
     p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
