@@ -261,6 +261,7 @@ def main():
             step()
             evs[i][1].record(stream)
             stages.append(hmg.hmg_stage_times())       # waits for this step's last stage event
+            redo = hmg.hmg_stage_counts()["vit_pair_redo"]
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -353,6 +354,7 @@ def main():
                        "flags_compaction_ms": round(st["msv_flags_compaction"], 4),
                        "vit_kernel_ms": round(vit_ms, 4), "vit_gcups": round(vit_gcups, 2) if vit_gcups else None,
                        "vit_flags_ms": round(st["vit_flags"], 4),
+                       "vit_pair_kernel": P.quant()["vit_pair_lanes"] > 0, "vit_s32_rescored": int(redo),
                        "survivors": int(ns_all), "survivor_frac": round(ns_all / max(n_all, 1), 5),
                        "survivor_residues": int(surv_all)},
             "roofline": roofline,

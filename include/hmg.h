@@ -71,7 +71,10 @@ typedef struct {
   const int16_t* tsc;               /* host [8][M]   BM MM IM DM MD MI II DD (clamped) */
   int msv_fast;                     /* 1: exact fast MSV kernel applies (bias < 66 + tbm) */
   int msv_lanes, msv_regs;          /* MSV kernel geometry: lanes per sequence G, s16x2 regs Q */
-  int vit_lanes, vit_nodes;         /* Viterbi kernel geometry: lanes per sequence, nodes per lane */
+  int vit_lanes, vit_nodes;         /* Viterbi s32 kernel geometry: lanes per sequence, nodes per lane */
+  int vit_pair_lanes, vit_pair_regs; /* s16x2 pair Viterbi kernel (two cells per register) in front of
+                                        the s32 kernel: lanes per sequence G, s16x2 registers Q per
+                                        cell type; 0 = not used for this profile */
 } hmg_quant;
 
 /* ---------------------------------------------------------------- profile */
@@ -190,6 +193,10 @@ int64_t hmg_kernel_launches(void);
  * Not thread-safe across concurrent calls (one global set of events). */
 hmg_status hmg_set_stage_timing(int enable);
 hmg_status hmg_stage_times(double* ms);
+/* With stage timing on: counts[0] = sequences of the most recent Viterbi stage that the s16x2
+ * pair kernel handed to the s32 kernel (outside its 16-bit window: strong hits, overflow
+ * neighbourhoods, all -inf rows), -1 if the pair kernel did not run.  Waits like hmg_stage_times. */
+hmg_status hmg_stage_counts(int64_t* counts);
 
 /* ---------------------------------------------------------------- host helpers (pure) */
 

@@ -56,6 +56,11 @@ struct VitArgs {
   int32_t* scratch;          // generic kernel: per-warp rows
   const uint8_t* done;       // skip sorted index s < ndone when done[s] (the pipeline long lane owns it)
   int64_t ndone;
+  // s16x2 pair kernel (vit_pair.cuh): per-sequence floor F = sat16(12000 + move(L) + tbm_min),
+  // safe = 32767 - (largest emission score); sequences outside the 16-bit window go to redo_list
+  int tbm_min, safe;
+  int32_t* redo_list;
+  unsigned long long* redo_count;
 };
 
 // Long-sequence lane (long.cu): chunked whole-warp MSV for the longest sequences and, in the
@@ -89,6 +94,10 @@ struct hmg_profile {
   int msv_fast = 0, msv_G = 0, msv_Q = 0;
   int vit_G = 0, vit_Q = 0, vit_generic = 0;
   int vit_W = 0;                    // >0: block-per-sequence kernel vit_cta_kernel<W, Q> (Q = vit_Q)
+  int pair_G = 0, pair_Q = 0;       // >0: s16x2 pair kernel vit_pair_kernel<G, Q> first, the above re-scores
+  int tbm_min = 0, rmax = 0;        // pair kernel window: min_k tBM_k, max(0, max_{x,k} rsc)
+  uint32_t* d_pair_rsc = nullptr;   // pair kernel tables: s16x2 emissions [kRows][G*Q] (chunk layout)
+  uint32_t* d_pair_tr = nullptr;    //                     s16x2 transitions [8][G][Q]
   // device tables
   uint32_t* d_msv_prof = nullptr;   // striped s16x2 emissions
   uint8_t* d_cost = nullptr;        // [kRows][M]
@@ -142,6 +151,8 @@ cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
 cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
 cudaError_t launch_vit_cta(int W, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_vit_pair(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+int vit_pair_q_max();
 size_t vit_cta_smem(int W, int Q);
 int long_msv_q(int QV);
 int msv_q_max(int G);

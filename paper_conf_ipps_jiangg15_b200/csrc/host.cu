@@ -34,6 +34,8 @@ struct StageTimer {
   int device = -1;
   cudaEvent_t ev[kStages + 1] = {};
   bool rec[kStages + 1] = {};
+  unsigned long long* h_redo = nullptr;   // pinned: sequences the pair Viterbi kernel handed back
+  bool redo_rec = false;
 } g_timer;
 std::mutex g_timer_mu;
 
@@ -44,6 +46,12 @@ void mark(int i, cudaStream_t st) {
 void mark_reset() {
   if (!g_timer.on) return;
   for (bool& r : g_timer.rec) r = false;
+  g_timer.redo_rec = false;
+}
+void stage_count_redo(const unsigned long long* d, cudaStream_t st) {
+  if (!g_timer.on || !g_timer.h_redo) return;
+  if (cudaMemcpyAsync(g_timer.h_redo, d, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st) == cudaSuccess)
+    g_timer.redo_rec = true;
 }
 
 constexpr double kLn2 = 0.693147180559945309417232121458176568;
@@ -300,6 +308,44 @@ void vit_tables_s16(const hmg_profile& p, int NT, int Q, std::vector<uint32_t>* 
       if (o < M) (*tr)[(size_t)t * NT * Q + o] = p.tsc[(size_t)t * M + o];
 }
 
+// pair-kernel tables (vit_pair.cuh): register q of lane z holds node z*Q+q+1 (low half) and
+// (z+G)*Q+q+1 (high half); emissions in the MSV chunk layout over Q words per lane, transitions
+// [8][G][Q]; padding nodes and nonexistent transitions are -32768 (the kernel's floor).
+void vit_pair_tables(const hmg_profile& p, int G, int Q, std::vector<uint32_t>* rsc, std::vector<uint32_t>* tr) {
+  const int M = p.M;
+  const int ROWW = Q * G;
+  rsc->assign(((size_t)kRows * ROWW + 3) / 4 * 4, 0u);
+  const int n4 = Q / 4, r = Q % 4;
+  auto word_index = [&](int z, int q) {
+    if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
+    int b = n4 * 4 * G;
+    int qq = q - n4 * 4;
+    if (r >= 2) {
+      if (qq < 2) return b + z * 2 + qq;
+      b += 2 * G;
+      qq -= 2;
+    }
+    return b + z;
+  };
+  auto r_of = [&](int x, int node) -> uint32_t {   // node 1-based
+    if (x >= kAlpha || node > M) return (uint16_t)(int16_t)kNegW;
+    return (uint16_t)p.rsc[(size_t)x * M + node - 1];
+  };
+  for (int x = 0; x < kRows; ++x)
+    for (int z = 0; z < G; ++z)
+      for (int q = 0; q < Q; ++q)
+        (*rsc)[(size_t)x * ROWW + word_index(z, q)] = r_of(x, z * Q + q + 1) | (r_of(x, (z + G) * Q + q + 1) << 16);
+  auto t_of = [&](int t, int node) -> uint32_t {
+    if (node > M) return (uint16_t)(int16_t)kNegW;
+    return (uint16_t)p.tsc[(size_t)t * M + node - 1];
+  };
+  tr->assign((size_t)8 * G * Q, 0u);
+  for (int t = 0; t < 8; ++t)
+    for (int z = 0; z < G; ++z)
+      for (int q = 0; q < Q; ++q)
+        (*tr)[(size_t)t * G * Q + z * Q + q] = t_of(t, z * Q + q + 1) | (t_of(t, (z + G) * Q + q + 1) << 16);
+}
+
 struct Scratch {
   std::vector<void*> bufs;
   cudaStream_t st;
@@ -506,30 +552,15 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
   return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 
-// Viterbi over sorted-order ids (list, device count) into raw_sorted.
-hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
-                   cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr,
-                   int64_t ndone = 0, bool marks = true) {
+// s32 Viterbi kernels (register / block / generic) for the profile's geometry
+hmg_status launch_vit_s32(const hmg_profile* p, VitArgs a, cudaStream_t st, Scratch& S) {
   cudaError_t e = cudaSuccess;
-  VitArgs a{};
-  a.words = db->d_words;
-  a.woff16 = db->d_woff16;
-  a.len = db->d_len;
-  a.nseq = db->nseq;
-  a.move = db->d_move;
   a.rsc = p->d_rsc;
   a.tr = p->d_tr;
-  a.M = p->M;
-  a.list = list;
-  a.nlist = nlist;
-  a.raw_sorted = raw_sorted;
-  a.done = done;
-  a.ndone = done ? ndone : 0;
   auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
   if (e) return cuda_status(e);
   if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
   a.counter = ctr;
-  if (marks) mark(3, st);
   if (!p->vit_generic && p->vit_W > 0) {
     int ok = 0;
     if ((e = launch_vit_cta(p->vit_W, p->vit_Q, a, st, &ok))) return cuda_status(e);
@@ -545,6 +576,58 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     a.scratch = scr;
     if ((e = launch_vit_generic(a, nwarps, st))) return cuda_status(e);
   }
+  return HMG_OK;
+}
+
+// Viterbi over sorted-order ids (list, device count) into raw_sorted.  With the s16x2 pair kernel
+// the sequences it cannot score exactly in its 16-bit window (vit_pair.cuh) are re-scored by the
+// s32 kernel from a device list (launched unconditionally; it exits at once when the list is empty).
+hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
+                   cudaStream_t st, int16_t* raw_sorted, Scratch& S, const uint8_t* done = nullptr,
+                   int64_t ndone = 0, bool marks = true, int64_t cap = -1) {
+  cudaError_t e = cudaSuccess;
+  VitArgs a{};
+  a.words = db->d_words;
+  a.woff16 = db->d_woff16;
+  a.len = db->d_len;
+  a.nseq = db->nseq;
+  a.move = db->d_move;
+  a.M = p->M;
+  a.list = list;
+  a.nlist = nlist;
+  a.raw_sorted = raw_sorted;
+  a.done = done;
+  a.ndone = done ? ndone : 0;
+  if (marks) mark(3, st);
+  hmg_status s = HMG_OK;
+  if (p->pair_G > 0) {
+    if (cap < 0) cap = db->nseq;                      // redo list capacity: entries of the id list
+    auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+    auto* redo = (int32_t*)S.get(sizeof(int32_t) * (size_t)std::max<int64_t>(cap, 1), &e);
+    if (e) return cuda_status(e);
+    if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+    VitArgs b = a;
+    b.rsc = reinterpret_cast<const int16_t*>(p->d_pair_rsc);
+    b.tr = reinterpret_cast<const int32_t*>(p->d_pair_tr);
+    b.counter = ctr;
+    b.tbm_min = p->tbm_min;
+    b.safe = 32767 - p->rmax;
+    b.redo_list = redo;
+    b.redo_count = ctr + 1;
+    int ok = 0;
+    if ((e = launch_vit_pair(p->pair_G, p->pair_Q, b, st, &ok))) return cuda_status(e);
+    if (!ok) return HMG_EUNSUPPORTED;
+    stage_count_redo(ctr + 1, st);
+    VitArgs r = a;                                   // re-score list: never in the long lane
+    r.list = redo;
+    r.nlist = reinterpret_cast<const int64_t*>(ctr + 1);
+    r.done = nullptr;
+    r.ndone = 0;
+    s = launch_vit_s32(p, r, st, S);
+  } else {
+    s = launch_vit_s32(p, a, st, S);
+  }
+  if (s != HMG_OK) return s;
   if (marks) mark(4, st);
   return HMG_OK;
 }
@@ -580,9 +663,12 @@ hmg_status hmg_set_stage_timing(int enable) {
     cudaGetDevice(&g_timer.device);
     for (auto& e : g_timer.ev)
       if (cudaEventCreate(&e) != cudaSuccess) return cuda_status(cudaGetLastError());
+    if (cudaMallocHost(&g_timer.h_redo, sizeof(unsigned long long)) != cudaSuccess)
+      return cuda_status(cudaGetLastError());
     g_timer.on = true;
   } else if (!enable && g_timer.on) {
     for (auto& e : g_timer.ev) cudaEventDestroy(e);
+    cudaFreeHost(g_timer.h_redo);
     g_timer = StageTimer();
   }
   return HMG_OK;
@@ -604,6 +690,19 @@ hmg_status hmg_stage_times(double* ms) {
     if (cudaEventElapsedTime(&t, g_timer.ev[i], g_timer.ev[i + 1]) == cudaSuccess) ms[i] = t;
     else cudaGetLastError();
   }
+  return HMG_OK;
+}
+
+hmg_status hmg_stage_counts(int64_t* counts) {
+  if (!counts) return HMG_EINVAL;
+  std::lock_guard<std::mutex> g(g_timer_mu);
+  if (!g_timer.on) return HMG_EINVAL;
+  counts[0] = -1;
+  int last = -1;
+  for (int i = kStages; i >= 0; --i)
+    if (g_timer.rec[i]) { last = i; break; }
+  if (last >= 0 && cudaEventSynchronize(g_timer.ev[last]) != cudaSuccess) return cuda_status(cudaGetLastError());
+  if (g_timer.redo_rec) counts[0] = (int64_t)*g_timer.h_redo;
   return HMG_OK;
 }
 
@@ -695,6 +794,29 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       }
     }
     p->vit_generic = p->vit_Q == 0 || env_int("HMG_VIT_GENERIC", 0);
+    // s16x2 pair kernel (vit_pair.cuh) in front of the s32 kernels: its 16-bit window must hold
+    // xN + move(L) + tBM_k .. 32767 for typical L, so entry scores and emissions must be moderate
+    int tmin = 32767, rmx = 0;
+    for (int k = 0; k < M; ++k) tmin = std::min(tmin, (int)p->tsc[k]);
+    for (int16_t v : p->rsc) rmx = std::max(rmx, (int)v);
+    p->tbm_min = tmin;
+    p->rmax = rmx;
+    if (tmin > -16384 && rmx < 8192 && !env_int("HMG_NO_VIT_PAIR", 0)) {
+      // lane-group size from the sweep (profiles/vit_pair_sweep_r01.jsonl): registers per lane
+      // (12 Q + ~30) set the warps per SM, so small Q (4-8) wins over fewer lanes per sequence
+      int g = M <= 64 ? 8 : M <= 128 ? 16 : 32;
+      const int o = env_int("HMG_VIT_PAIR_G", 0);
+      if (o == 8 || o == 16 || o == 32) g = o;
+      int q = (M + 2 * g - 1) / (2 * g);
+      while (q > vit_pair_q_max() && g < 32) {
+        g *= 2;
+        q = (M + 2 * g - 1) / (2 * g);
+      }
+      if (q <= vit_pair_q_max()) {
+        p->pair_G = g;
+        p->pair_Q = q;
+      }
+    }
   }
   if (device < 0) {
     *out = p;
@@ -741,6 +863,12 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       st = upload(&p->d_rsc, r.data(), r.size());
       if (st == HMG_OK) st = upload(&p->d_tr, t.data(), t.size());
     }
+  }
+  if (st == HMG_OK && tsc && p->pair_G > 0) {
+    std::vector<uint32_t> r, t;
+    vit_pair_tables(*p, p->pair_G, p->pair_Q, &r, &t);
+    st = upload(&p->d_pair_rsc, r.data(), r.size());
+    if (st == HMG_OK) st = upload(&p->d_pair_tr, t.data(), t.size());
   }
   if (st == HMG_OK && tsc && M <= 512 && !env_int("HMG_NO_LONG_LANE", 0)) {
     const int QV = (M + 31) / 32;
@@ -844,6 +972,8 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->msv_regs = p->msv_Q;
   q->vit_lanes = p->vit_generic ? 32 : p->vit_G;   // block kernel: 32 * warps
   q->vit_nodes = p->vit_generic ? 0 : p->vit_Q;
+  q->vit_pair_lanes = p->pair_G;
+  q->vit_pair_regs = p->pair_Q;
   return HMG_OK;
 }
 
@@ -858,6 +988,8 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_long_msv);
     cudaFree(p->d_long_rsc);
     cudaFree(p->d_long_tr);
+    cudaFree(p->d_pair_rsc);
+    cudaFree(p->d_pair_tr);
     cudaFree(p->thr_msv.d);
     cudaFree(p->thr_vit.d);
     cudaGetLastError();
@@ -1091,7 +1223,7 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
       nmax = n;
     }
     mark_reset();
-    hmg_status s = run_vit(p, db, list, nl, st, raw_sorted, S);
+    hmg_status s = run_vit(p, db, list, nl, st, raw_sorted, S, nullptr, 0, true, nmax);
     if (s != HMG_OK) return s;
     e = vit_finish(raw_sorted, list, nl, nmax, db->d_len, db->d_order, thr, raw, pass, nullptr, st);
     mark(5, st);

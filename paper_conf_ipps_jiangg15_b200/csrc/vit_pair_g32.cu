@@ -1,0 +1,17 @@
+// Instantiations of vit_pair_kernel<32, Q> for Q = 1..16.
+#include "vit_pair.cuh"
+
+namespace hmg {
+namespace {
+template <int Q>
+const void* pick(int q) {
+  if constexpr (Q > 16) {
+    return nullptr;
+  } else {
+    if (q == Q) return reinterpret_cast<const void*>(&vit_pair_kernel<32, Q>);
+    return pick<Q + 1>(q);
+  }
+}
+}  // namespace
+const void* vit_pair_ptr_g32(int q) { return pick<1>(q); }
+}  // namespace hmg

@@ -30,7 +30,8 @@ class hmg_quant(ctypes.Structure):
                 ("scale_b", c_f), ("base_w", c_int), ("xw_e", c_int), ("ddbound_w", c_int), ("scale_w", c_f),
                 ("cost", ctypes.POINTER(ctypes.c_uint8)), ("rsc", ctypes.POINTER(ctypes.c_int16)),
                 ("tsc", ctypes.POINTER(ctypes.c_int16)), ("msv_fast", c_int), ("msv_lanes", c_int),
-                ("msv_regs", c_int), ("vit_lanes", c_int), ("vit_nodes", c_int)]
+                ("msv_regs", c_int), ("vit_lanes", c_int), ("vit_nodes", c_int),
+                ("vit_pair_lanes", c_int), ("vit_pair_regs", c_int)]
 
 
 # name -> (restype, argtypes), exactly the declarations of include/hmg.h
@@ -59,6 +60,7 @@ SIGNATURES = {
     "hmg_calibrate": (c_int, [c_p, c_int, c_int, ctypes.c_uint64, c_d, c_p]),
     "hmg_set_stage_timing": (c_int, [c_int]),
     "hmg_stage_times": (c_int, [c_p]),
+    "hmg_stage_counts": (c_int, [c_p]),
 }
 
 
@@ -278,6 +280,14 @@ def hmg_stage_times() -> dict:
     ms = np.zeros(5, dtype=np.float64)
     _check(lib().hmg_stage_times(_np_ptr(ms)), "hmg_stage_times")
     return dict(zip(STAGES, ms.tolist()))
+
+
+def hmg_stage_counts() -> dict:
+    """Counts of the most recent call (stage timing on): sequences the s16x2 pair Viterbi kernel
+    handed back to the s32 kernel (-1: the pair kernel did not run)."""
+    c = np.zeros(1, dtype=np.int64)
+    _check(lib().hmg_stage_counts(_np_ptr(c)), "hmg_stage_counts")
+    return {"vit_pair_redo": int(c[0])}
 
 
 # ------------------------------------------------------------------------ convenience

@@ -172,7 +172,12 @@ VMS = [1, 2, 3, 4, 5, 8, 9, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 
 
 @pytest.mark.parametrize("M", VMS)
 @pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
-def test_vit_model_lengths(M, dd):
+@pytest.mark.parametrize("pair", [True, False])
+def test_vit_model_lengths(M, dd, pair, monkeypatch):
+    """pair: the s16x2 pair kernel (+ s32 re-scoring of what leaves its window); otherwise the
+    s32 kernels alone (HMG_NO_VIT_PAIR)."""
+    if not pair:
+        monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M + int(dd[0]))
     prof = synth.make_profile(M, 8000 + M, dd=dd)
     n = 40 if M <= 600 else 12
@@ -199,6 +204,78 @@ def test_vit_long_delete_chains(M):
     dsq, off = _db_from(seqs)
     got, _ = _vit_gpu(msc, tsc, dsq, off)
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
+
+
+@pytest.mark.parametrize("pair", [True, False])
+def test_vit_long_delete_chains_s32(pair, monkeypatch):
+    """The delete-chain profiles above have -inf entry below node 1, so the pair kernel does not
+    apply; here entry is finite everywhere but weak, so the pair kernel's Lazy-F (carries through
+    both halves of every register, lane G-1 low -> lane 0 high) decides the score."""
+    if not pair:
+        monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
+    for M in (3, 20, 64, 130, 300, 500, 700, 1000):
+        rng = np.random.default_rng(M + 17)
+        msc = np.full((M, 29), -6.0, np.float32)
+        msc[0, 0] = 4.0
+        msc[M - 1, 1] = 4.0
+        msc[M // 2, 2] = 3.0
+        tsc = np.log(rng.uniform(0.05, 1.0, size=(M, 8))).astype(np.float32)
+        tsc[:, 7] = np.log(rng.uniform(0.8, 0.999, size=M))
+        tsc[:, 0] = np.log(1e-4 / M)
+        tsc[0, 0] = np.log(0.5)
+        tsc[0, 1:4] = -np.inf
+        tsc[M - 1, 4:8] = -np.inf
+        seqs = [np.array([0, 1], np.uint8), np.array([0, 2, 1], np.uint8), np.array([0, 1, 0, 1], np.uint8)]
+        seqs += [synth.random_dsq(rng, int(L), 3) for L in rng.integers(1, 60, size=30)]
+        dsq, off = _db_from(seqs)
+        got, p = _vit_gpu(msc, tsc, dsq, off)
+        assert (p.quant()["vit_pair_lanes"] > 0) == (pair and M <= 1024), M
+        assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off)), M
+
+
+@pytest.mark.parametrize("G", [8, 16, 32])
+@pytest.mark.parametrize("M", [10, 100, 257, 600])
+def test_vit_pair_every_lane_group(G, M, monkeypatch):
+    monkeypatch.setenv("HMG_VIT_PAIR_G", str(G))
+    rng = np.random.default_rng(G + M)
+    prof = synth.make_profile(M, 300 + M + G, dd=(1.0, 9.0))
+    dsq, off = _ragged_db(rng, n=70, alphabet=29, lmax=350)
+    got, p = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+    q = p.quant()
+    assert q["vit_pair_lanes"] >= G and 2 * q["vit_pair_lanes"] * q["vit_pair_regs"] >= M
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off))
+
+
+def test_vit_pair_window_exits():
+    """Sequences the pair kernel hands to the s32 kernel: strong planted hits (cells above the
+    16-bit window), overflow, gap-only sequences (every row floored); and long sequences whose
+    floor F is low.  Scores stay bit-exact and some sequences are re-scored."""
+    rng = np.random.default_rng(8)
+    M = 180
+    prof = synth.make_profile(M, 818)
+    msc = prof.msc.copy()
+    best = np.argmax(msc[:, :20], axis=1).astype(np.uint8)
+    seqs = []
+    for i in range(120):
+        L = int(rng.integers(5, 900)) if i % 10 else int(rng.integers(3000, 9000))
+        d = synth.random_dsq(rng, L)
+        if i % 4 == 0:                         # best-path prefixes: below, inside and above the window
+            seg = best[: min(L, int(rng.integers(5, M + 1)))]
+            a = int(rng.integers(0, L - len(seg) + 1))
+            d[a:a + len(seg)] = seg
+        seqs.append(d)
+    seqs += [np.full(L, 20, np.uint8) for L in (1, 5, 40)] + [np.array([27, 28, 20, 27], np.uint8)]
+    dsq, off = _db_from(seqs)
+    hmg.hmg_set_stage_timing(True)
+    try:
+        got, p = _vit_gpu(msc, prof.tsc, dsq, off)
+        redo = hmg.hmg_stage_counts()["vit_pair_redo"]
+    finally:
+        hmg.hmg_set_stage_timing(False)
+    want = oracle.vit_db(oracle.VitProfile(msc, prof.tsc), dsq, off)
+    assert p.quant()["vit_pair_lanes"] > 0
+    assert np.array_equal(got, want)
+    assert (want == 32767).sum() > 0 and redo >= 4
 
 
 def test_vit_overflow_and_minus_inf():
@@ -335,6 +412,7 @@ def test_vit_block_kernel(M, dd, monkeypatch):
     """Block-per-sequence Viterbi (W warps per row, cross-warp Lazy-F through shared memory);
     forced for small M with HMG_VIT_CTA, used by default above M = 512."""
     monkeypatch.setenv("HMG_VIT_CTA", "1")
+    monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M * 3 + int(dd[1]))
     prof = synth.make_profile(M, 9000 + M, dd=dd)
     n = 30 if M <= 1100 else 10
@@ -349,6 +427,7 @@ def test_vit_block_kernel(M, dd, monkeypatch):
 def test_vit_block_kernel_delete_chains(M, monkeypatch):
     """D->D chains that cross every warp boundary of the block (cross-warp Lazy-F rounds)."""
     monkeypatch.setenv("HMG_VIT_CTA", "1")
+    monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M + 5)
     msc = np.full((M, 29), -6.0, np.float32)
     msc[0, 0] = 4.0
