@@ -105,7 +105,9 @@ struct hmg_profile {
   int32_t* d_tr = nullptr;          // Viterbi transitions (layout per kernel)
   size_t msv_prof_bytes = 0, vit_rsc_bytes = 0, vit_tr_bytes = 0;
   // pipeline long lane (whole-warp MSV + Viterbi), available when M <= 512
-  int long_QV = 0;
+  int long_QV = 0;                  // >0: long lane available; Viterbi regs per lane (s32 nodes or pair regs)
+  int long_QL = 0;                  // whole-warp MSV registers of the chunked long-lane MSV
+  bool long_pair = false;           // long-lane Viterbi uses the pair lane and d_pair_* (G = 32)
   uint32_t* d_long_msv = nullptr;
   int32_t* d_long_rsc = nullptr;
   int32_t* d_long_tr = nullptr;
@@ -148,13 +150,13 @@ cudaError_t launch_msv_fast(int G, int Q, const MsvArgs& a, cudaStream_t st, int
 cudaError_t launch_msv_exact(const MsvArgs& a, int nwarps, cudaStream_t st);
 cudaError_t launch_vit_reg(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_vit_generic(const VitArgs& a, int nwarps, cudaStream_t st);
-cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int* ok);
-cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
+cudaError_t launch_pipe_long_msv(int QL, const LongArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_pipe_long_vit(int QV, bool pair, const LongArgs& a, int nblocks, cudaStream_t st, int* ok);
 cudaError_t launch_vit_cta(int W, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 cudaError_t launch_vit_pair(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 int vit_pair_q_max();
 size_t vit_cta_smem(int W, int Q);
-int long_msv_q(int QV);
+int long_msv_q(int M);
 int msv_q_max(int G);
 int msv_table_words(int G, int Q);   // MsvLayout<G, Q>::WORDS
 int vit_q_max(int G);

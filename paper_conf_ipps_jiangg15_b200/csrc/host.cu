@@ -548,7 +548,7 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
   la.chunk_done = cdone;
   la.counter = lctr;
   int ok = 0;
-  if ((e = launch_pipe_long_msv(p->long_QV, la, st, &ok))) return cuda_status(e);
+  if ((e = launch_pipe_long_msv(p->long_QL, la, st, &ok))) return cuda_status(e);
   return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 
@@ -870,16 +870,31 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     st = upload(&p->d_pair_rsc, r.data(), r.size());
     if (st == HMG_OK) st = upload(&p->d_pair_tr, t.data(), t.size());
   }
-  if (st == HMG_OK && tsc && M <= 512 && !env_int("HMG_NO_LONG_LANE", 0)) {
-    const int QV = (M + 31) / 32;
-    auto tm = msv_table(*p, 32, long_msv_q(QV));
-    std::vector<uint32_t> r;
-    std::vector<int32_t> t;
-    vit_tables(*p, 32, QV, &r, &t);
+  // pipeline long lane: whole-warp Viterbi with the pair lane (the pair tables when G = 32, models
+  // up to 1024 nodes) or the s32 latency lane (models up to 512 nodes)
+  const bool lpair = p->pair_G == 32 && !env_int("HMG_LONG_S32", 0);
+  if (st == HMG_OK && tsc && (lpair || M <= 512) && !env_int("HMG_NO_LONG_LANE", 0)) {
+    const int QL = long_msv_q(M);
+    auto tm = msv_table(*p, 32, QL);
     st = upload(&p->d_long_msv, tm.data(), tm.size());
-    if (st == HMG_OK) st = upload(reinterpret_cast<uint32_t**>(&p->d_long_rsc), r.data(), r.size());
-    if (st == HMG_OK) st = upload(&p->d_long_tr, t.data(), t.size());
-    if (st == HMG_OK) p->long_QV = QV;
+    if (lpair) {
+      if (st == HMG_OK) {
+        p->long_QV = p->pair_Q;
+        p->long_pair = true;
+        p->long_QL = QL;
+      }
+    } else {
+      const int QV = (M + 31) / 32;
+      std::vector<uint32_t> r;
+      std::vector<int32_t> t;
+      vit_tables(*p, 32, QV, &r, &t);
+      if (st == HMG_OK) st = upload(reinterpret_cast<uint32_t**>(&p->d_long_rsc), r.data(), r.size());
+      if (st == HMG_OK) st = upload(&p->d_long_tr, t.data(), t.size());
+      if (st == HMG_OK) {
+        p->long_QV = QV;
+        p->long_QL = QL;
+      }
+    }
   }
   if (st != HMG_OK) {
     hmg_profile_destroy(p);
@@ -1260,7 +1275,8 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     // pipeline long lane (long.cu): chunked MSV of the longest sequences on the whole GPU, then
     // their Viterbi filter on SMs held alone by pipe_long_vit_kernel while the main MSV kernel
     // (programmatic dependent launch) fills the other SMs
-    const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && !p->vit_generic && p->vit_W == 0 &&
+    const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 &&
+                           (p->long_pair || (!p->vit_generic && p->vit_W == 0)) &&
                            !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
     auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
@@ -1276,8 +1292,10 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       la.v.len = db->d_len;
       la.v.nseq = n;
       la.v.move = db->d_move;
-      la.v.rsc = reinterpret_cast<const int16_t*>(p->d_long_rsc);
-      la.v.tr = p->d_long_tr;
+      la.v.rsc = reinterpret_cast<const int16_t*>(p->long_pair ? (void*)p->d_pair_rsc : (void*)p->d_long_rsc);
+      la.v.tr = reinterpret_cast<const int32_t*>(p->long_pair ? (void*)p->d_pair_tr : (void*)p->d_long_tr);
+      la.v.tbm_min = p->tbm_min;
+      la.v.safe = 32767 - p->rmax;
       la.v.M = p->M;
       la.v.raw_sorted = vraw_sorted;
       la.thr = tm;
@@ -1285,7 +1303,7 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
       int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
       nb = env_int("HMG_PIPE_LONG_SMS", nb);
       int ok = 0;
-      if ((e = launch_pipe_long_vit(p->long_QV, la, nb, st, &ok))) return cuda_status(e);
+      if ((e = launch_pipe_long_vit(p->long_QV, p->long_pair, la, nb, st, &ok))) return cuda_status(e);
       if (!ok) return HMG_EUNSUPPORTED;
     }
     s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV

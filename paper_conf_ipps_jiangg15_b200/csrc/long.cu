@@ -16,19 +16,23 @@
 //   pipe_long_vit_kernel<QV>   the Viterbi filter (latency variant of VitLane) of the long
 //                              sequences that pass, on SMs it holds alone, while the main MSV
 //                              kernel (programmatic dependent launch) fills the other SMs
-//                              (hmg_pipeline).
+//                              (hmg_pipeline);
+//   pipe_long_vpair_kernel<Q>  the same with the s16x2 pair lane (vit_pair.cuh), whole warp,
+//                              for models up to 1024 nodes; sequences it cannot score in its
+//                              16-bit window are left to the main Viterbi stage (owned = 0).
 #include <cuda_runtime.h>
 
 #include <algorithm>
 
 #include "msv.cuh"
 #include "vit.cuh"
+#include "vit_pair.cuh"
 
 namespace hmg {
 
 // whole-warp MSV registers that cover a model of up to 32*QV nodes (2*32*QL >= 32*QV + 1)
-__host__ __device__ constexpr int long_msv_q_of(int QV) { return (32 * QV + 1 + 63) / 64; }
-int long_msv_q(int QV) { return long_msv_q_of(QV); }
+// whole-warp MSV registers for a model of M nodes: 2 * 32 * QL >= M + 1
+int long_msv_q(int M) { return (M + 1 + 63) / 64; }
 
 template <int QL>
 __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
@@ -150,7 +154,68 @@ __global__ void __launch_bounds__(128) pipe_long_vit_kernel(const LongArgs A) {
   }
 }
 
+template <int Q>
+__global__ void __launch_bounds__(128) pipe_long_vpair_kernel(const LongArgs A) {
+  asm volatile("griddepcontrol.launch_dependents;");
+  constexpr int WV = kRows * Q * 32;
+  extern __shared__ uint4 smem4[];
+  {
+    const uint4* s1 = reinterpret_cast<const uint4*>(A.v.rsc);
+    for (int i = threadIdx.x; i < WV / 4; i += blockDim.x) smem4[i] = s1[i];
+  }
+  __syncthreads();
+  const uint32_t* smv = reinterpret_cast<const uint32_t*>(smem4);
+  const uint32_t* tr = reinterpret_cast<const uint32_t*>(A.v.tr);
+  const int lane = threadIdx.x & 31;
+  VitPairLane<32, Q> V;
+  V.load(tr, lane);
+  for (;;) {
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(A.counter + 1, 1ull);
+    b = __shfl_sync(0xffffffffu, b, 0);
+    if ((long long)b >= A.nlong) break;
+    const int j = (int)b;
+    if (!A.owned[j]) continue;                   // 254: the exact re-score + main stage decide
+    const int raw = A.m.raw[j];
+    const int L = A.m.len[j];
+    if (!(raw == 255 || raw >= (int)A.thr[L])) continue;       // MSV pass flag (reading R25)
+    const uint32_t* wp = A.v.words + (size_t)A.v.woff16[j] * 4;
+    V.start(tr, lane, A.v.move[L], A.v.tbm_min, A.v.safe, true, 0xffffffffu);
+    ResStream rs;
+    rs.init(wp, (L + 5) / 6);
+    for (int iq = 0; iq < rs.nq; ++iq) {                        // Alg 2 row loop
+      uint4 w4 = rs.next(iq);
+#pragma unroll 1
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t w = w4.x;
+        w4.x = w4.y;
+        w4.y = w4.z;
+        w4.z = w4.w;
+#pragma unroll
+        for (int jj = 0; jj < 6; ++jj) {
+          const int x = (w >> (5 * jj)) & 31;
+          V.row(smv + x * (Q * 32), tr, lane, 0xffffffffu);
+        }
+      }
+    }
+    const int vraw = V.finish();
+    if (lane == 0) {
+      if (vraw >= -32768) A.v.raw_sorted[j] = (int16_t)vraw;
+      else A.owned[j] = 0;                       // outside the window: the main stage scores it
+    }
+  }
+}
+
 namespace {
+template <int Q>
+const void* pick_vpair(int q) {
+  if constexpr (Q > 16) {
+    return nullptr;
+  } else {
+    if (q == Q) return reinterpret_cast<const void*>(&pipe_long_vpair_kernel<Q>);
+    return pick_vpair<Q + 1>(q);
+  }
+}
 template <int QV>
 const void* pick_vit(int q) {
   if constexpr (QV > 16) {
@@ -162,7 +227,7 @@ const void* pick_vit(int q) {
 }
 template <int QL>
 const void* pick_msv(int q) {
-  if constexpr (QL > 9) {   // QV <= 16 -> QL <= 9
+  if constexpr (QL > 17) {   // models up to 1024 nodes
     return nullptr;
   } else {
     if (q == QL) return reinterpret_cast<const void*>(&pipe_long_msv_kernel<QL>);
@@ -171,8 +236,7 @@ const void* pick_msv(int q) {
 }
 }  // namespace
 
-cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int* ok) {
-  const int QL = long_msv_q_of(QV);
+cudaError_t launch_pipe_long_msv(int QL, const LongArgs& a, cudaStream_t st, int* ok) {
   const void* fn = pick_msv<1>(QL);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
@@ -194,8 +258,8 @@ cudaError_t launch_pipe_long_msv(int QV, const LongArgs& a, cudaStream_t st, int
 }  // namespace hmg
 
 namespace hmg {
-cudaError_t launch_pipe_long_vit(int QV, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
-  const void* fn = pick_vit<1>(QV);
+cudaError_t launch_pipe_long_vit(int QV, bool pair, const LongArgs& a, int nblocks, cudaStream_t st, int* ok) {
+  const void* fn = pair ? pick_vpair<1>(QV) : pick_vit<1>(QV);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
   const size_t need = (size_t)kRows * QV * 32 * 4;

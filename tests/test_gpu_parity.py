@@ -445,16 +445,22 @@ def test_vit_block_kernel_delete_chains(M, monkeypatch):
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
 
 
-@pytest.mark.parametrize("chunk,sms", [(1032, "0"), (60, "0"), (1032, "2")])
-def test_pipeline_long_lane(chunk, sms, monkeypatch):
+@pytest.mark.parametrize("chunk,sms,M,lane", [(1032, "0", 120, "s32"), (60, "0", 120, "s32"),
+                                               (1032, "2", 120, "s32"), (1032, "0", 300, "pair"),
+                                               (60, "3", 300, "s32"), (1032, "0", 700, "pair"),
+                                               (200, "2", 1000, "pair")])
+def test_pipeline_long_lane(chunk, sms, M, lane, monkeypatch):
     """The pipeline long lane: sequences longer than max(1500, 8 x mean) get chunked MSV (rows
-    from the empty state M rows early) and whole-warp Viterbi on a side stream.  Strong planted
-    hits in some long sequences force the sequential fallback (a chunk sees a J->B row)."""
+    from the empty state M rows early) and whole-warp Viterbi on SMs held alone (the s32 latency
+    lane, or the s16x2 pair lane for models of 129..1024 nodes).  Strong planted hits in some
+    long sequences force the sequential fallback (a chunk sees a J->B row)."""
     monkeypatch.setenv("HMG_PIPE_CHUNK", str(chunk))
     if sms != "0":
         monkeypatch.setenv("HMG_PIPE_LONG_SMS", sms)
+    if lane == "s32":
+        monkeypatch.setenv("HMG_LONG_S32", "1")
     rng = np.random.default_rng(42)
-    prof = synth.make_profile(120, 4242)
+    prof = synth.make_profile(M, 4242 + M)
     best = np.argmax(prof.msc[:, :20], axis=1).astype(np.uint8)
     seqs = []
     for i in range(300):
@@ -468,3 +474,26 @@ def test_pipeline_long_lane(chunk, sms, monkeypatch):
     dsq, off = _db_from(seqs)
     ns = _check_pipeline(prof, dsq, off, F1=0.02, F2=1e-3)
     assert ns >= 10
+
+
+@pytest.mark.parametrize("M", [130, 300, 451, 641, 1000])
+def test_pipeline_many_survivors(M):
+    """Pipeline with the pair Viterbi kernel at every MSV lane-group geometry: loose F1 sends many
+    sequences to the Viterbi stage; planted hits and gap-only sequences take the overflow /
+    re-score paths."""
+    rng = np.random.default_rng(M + 77)
+    prof = synth.make_profile(M, 5000 + M)
+    best = np.argmax(prof.msc[:, :20], axis=1).astype(np.uint8)
+    seqs = []
+    for i in range(700):
+        L = int(rng.integers(1, 900))
+        d = synth.random_dsq(rng, L, 20)
+        if i % 37 == 0:
+            seg = best[: min(L, int(rng.integers(5, M + 1)))]
+            a = int(rng.integers(0, L - len(seg) + 1))
+            d[a:a + len(seg)] = seg
+        seqs.append(d)
+    seqs += [np.full(L, 20, np.uint8) for L in (3, 60)]
+    dsq, off = _db_from(seqs)
+    ns = _check_pipeline(prof, dsq, off, F1=0.3, F2=0.05)
+    assert ns > 100
