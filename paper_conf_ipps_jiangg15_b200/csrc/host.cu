@@ -615,7 +615,11 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     b.redo_list = redo;
     b.redo_count = ctr + 1;
     int ok = 0;
-    if ((e = launch_vit_pair(p->pair_G, p->pair_Q, b, st, &ok))) return cuda_status(e);
+    if (p->pair_W > 0) {
+      if ((e = launch_vit_cpair(p->pair_W, p->pair_SG, p->pair_Q, b, st, &ok))) return cuda_status(e);
+    } else {
+      if ((e = launch_vit_pair(p->pair_G, p->pair_Q, b, st, &ok))) return cuda_status(e);
+    }
     if (!ok) return HMG_EUNSUPPORTED;
     stage_count_redo(ctr + 1, st);
     VitArgs r = a;                                   // re-score list: never in the long lane
@@ -812,9 +816,35 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
         g *= 2;
         q = (M + 2 * g - 1) / (2 * g);
       }
-      if (q <= vit_pair_q_max()) {
+      if (q <= vit_pair_q_max() && !env_int("HMG_VIT_PAIR_CTA", 0)) {
         p->pair_G = g;
         p->pair_Q = q;
+      } else {   // long models: block-per-sequence pair kernel, W warps on one DP row
+        // W warps per sequence and SG sequences per block from the sweep on the config-4 shape
+        // (profiles/vit_cpair_sweep_r01.jsonl): 2 warps x 16 registers per thread, 2 sequences
+        // per block sharing the table, up to M = 2048; wider rows above
+        int W = M <= 2048 ? 2 : 4, SG = M <= 2048 ? 2 : 1;
+        const int wo = env_int("HMG_VIT_PAIR_W", 0);
+        if (wo == 2 || wo == 4 || wo == 8 || wo == 16) {
+          W = wo;
+          SG = W == 2 ? 2 : W == 4 ? 3 : W == 8 ? 2 : 1;
+        }
+        SG = env_int("HMG_VIT_PAIR_SG", SG);
+        int qq = std::max(2, (M + 64 * W - 1) / (64 * W));
+        while (!vit_cpair_available(W, SG, qq) && W < 16) {   // models too long for W warps
+          W *= 2;
+          SG = 1;
+          qq = std::max(2, (M + 64 * W - 1) / (64 * W));
+        }
+        int smax = 0;
+        if (device >= 0) cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+        else smax = 227 * 1024;
+        if (vit_cpair_available(W, SG, qq) && vit_cpair_smem(W, SG, qq) <= (size_t)smax) {
+          p->pair_W = W;
+          p->pair_SG = SG;
+          p->pair_G = 32 * W;
+          p->pair_Q = qq;
+        }
       }
     }
   }
@@ -872,7 +902,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   }
   // pipeline long lane: whole-warp Viterbi with the pair lane (the pair tables when G = 32, models
   // up to 1024 nodes) or the s32 latency lane (models up to 512 nodes)
-  const bool lpair = p->pair_G == 32 && !env_int("HMG_LONG_S32", 0);
+  const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !env_int("HMG_LONG_S32", 0);
   if (st == HMG_OK && tsc && (lpair || M <= 512) && !env_int("HMG_NO_LONG_LANE", 0)) {
     const int QL = long_msv_q(M);
     auto tm = msv_table(*p, 32, QL);

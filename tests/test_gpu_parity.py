@@ -497,3 +497,50 @@ def test_pipeline_many_survivors(M):
     dsq, off = _db_from(seqs)
     ns = _check_pipeline(prof, dsq, off, F1=0.3, F2=0.05)
     assert ns > 100
+
+
+@pytest.mark.parametrize("M", [2, 3, 64, 300, 513, 1024, 1025, 1500, 2048, 2600, 4000])
+@pytest.mark.parametrize("W", [2, 4, 8, 16])
+def test_vit_block_pair_kernel(M, W, monkeypatch):
+    """Block-per-sequence pair kernel (W warps per row, 2 cells per register, closed-form carries
+    across virtual warps); forced for small M with HMG_VIT_PAIR_CTA, used by default above 1024."""
+    monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
+    monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
+    rng = np.random.default_rng(M * 7 + W)
+    for dd in [(7.0, 3.0), (1.0, 9.0)]:
+        prof = synth.make_profile(M, 9100 + M + W, dd=dd)
+        n = 24 if M <= 1100 else 8
+        dsq, off = _ragged_db(rng, n=n, alphabet=29, lmax=250)
+        got, p = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+        q = p.quant()
+        assert q["vit_pair_lanes"] >= 32 * W and 2 * q["vit_pair_lanes"] * q["vit_pair_regs"] >= M
+        assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)), dd
+
+
+@pytest.mark.parametrize("W", [2, 4, 8, 16])
+def test_vit_block_pair_delete_chains_and_exits(W, monkeypatch):
+    """D->D chains across every virtual-warp boundary (low halves -> high halves), strong hits that
+    re-base the window or overflow, and gap-only sequences handed to the s32 kernel."""
+    monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
+    monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
+    for M in (40, 700, 2000):
+        rng = np.random.default_rng(M + W)
+        msc = np.full((M, 29), -6.0, np.float32)
+        msc[0, 0] = 4.0
+        msc[M - 1, 1] = 4.0
+        msc[M // 2, 2] = 3.0
+        msc[:, 3] = 2.5                              # residue 3 scores everywhere: strong hits
+        tsc = np.log(rng.uniform(0.05, 1.0, size=(M, 8))).astype(np.float32)
+        tsc[:, 7] = np.log(rng.uniform(0.9, 0.9999, size=M))
+        tsc[:, 0] = np.log(1e-4 / M)
+        tsc[0, 0] = np.log(0.5)
+        tsc[0, 1:4] = -np.inf
+        tsc[M - 1, 4:8] = -np.inf
+        seqs = [np.array([0, 1], np.uint8), np.array([0, 2, 1], np.uint8), np.array([0, 1, 0, 2, 1], np.uint8)]
+        seqs += [synth.random_dsq(rng, int(L), 3) for L in rng.integers(1, 40, size=12)]
+        seqs += [np.full(L, 3, np.uint8) for L in (5, 30, 200)] + [np.full(7, 20, np.uint8)]
+        dsq, off = _db_from(seqs)
+        got, p = _vit_gpu(msc, tsc, dsq, off)
+        assert p.quant()["vit_pair_lanes"] >= 32 * W
+        want = oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off)
+        assert np.array_equal(got, want), M

@@ -27,7 +27,7 @@ peaks = json.load(open(os.path.join(os.path.dirname(os.path.dirname(os.path.absp
 f_sm = float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
 P_INT = 64 * 148 * f_sm          # ALU-pipe lane-ops/s
 msv_roof = P_INT / 0.75          # cells/s at 0.75 ALU ops per cell
-vit_roof = P_INT / 9.5           # cells/s at 9.5 ALU ops per cell
+vit_roof = P_INT / 4.25          # cells/s at 4.25 ALU ops per cell (s16x2 pair encoding, DESIGN 4.6)
 
 
 def timed(fn, reps=3):
@@ -107,12 +107,14 @@ for cfg in which:
         P = hmg.Profile(prof.msc, prof.tsc)
         D = hmg.Database(dsq, off)
         vraw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
-        ms, st = timed(lambda: hmg.hmg_viterbi(P, D, vraw), reps=1)
+        ms, st = timed(lambda: hmg.hmg_viterbi(P, D, vraw), reps=2)
         g = 2048 * D.residues / (st["vit_kernel"] * 1e-3)
         q = P.quant()
         report(4, 2048, D, ms, st, {"stage": "viterbi_all", "vit_gcups": round(g / 1e9, 1),
                                     "vit_roof_frac": round(g / vit_roof, 3),
-                                    "kernel": "vit_cta_kernel<%d,%d>" % (q["vit_lanes"] // 32, q["vit_nodes"])})
+                                    "kernel": ("vit_cpair_kernel<W=%d, Q=%d>" % (q["vit_pair_lanes"] // 32, q["vit_pair_regs"])
+                                               if q["vit_pair_lanes"] else
+                                               "vit_cta_kernel<%d,%d>" % (q["vit_lanes"] // 32, q["vit_nodes"]))})
     elif cfg == 5:
         c = synth.CONFIGS[5]
         L = synth.make_lengths(c["N"], c["mu_ln"], c["sigma"], c["dseed"])
