@@ -618,7 +618,7 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     if (p->pair_W > 0) {
       if ((e = launch_vit_cpair(p->pair_W, p->pair_SG, p->pair_Q, b, st, &ok))) return cuda_status(e);
     } else {
-      if ((e = launch_vit_pair(p->pair_G, p->pair_Q, b, st, &ok))) return cuda_status(e);
+      if ((e = launch_vit_pair(p->pair_G, p->pair_Q, p->pair_scan, b, st, &ok))) return cuda_status(e);
     }
     if (!ok) return HMG_EUNSUPPORTED;
     stage_count_redo(ctr + 1, st);
@@ -819,6 +819,12 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       if (q <= vit_pair_q_max() && !env_int("HMG_VIT_PAIR_CTA", 0)) {
         p->pair_G = g;
         p->pair_Q = q;
+        // Lazy-F by max-plus scan (f1) when D->D chains are long: its cost does not depend on the
+        // profile, the vote-terminated passes win on typical ones (profiles/vit_scan_f1_r01.jsonl)
+        double pdd = 0.0;
+        for (int k = 0; k + 1 < M; ++k) pdd += std::exp((double)tsc[(size_t)k * 8 + 7]);
+        pdd = M > 1 ? pdd / (M - 1) : 0.0;
+        p->pair_scan = g == 32 && env_int("HMG_VIT_SCAN", pdd > 0.6 ? 1 : 0);
       } else {   // long models: block-per-sequence pair kernel, W warps on one DP row
         // W warps per sequence and SG sequences per block from the sweep on the config-4 shape
         // (profiles/vit_cpair_sweep_r01.jsonl): 2 warps x 16 registers per thread, 2 sequences

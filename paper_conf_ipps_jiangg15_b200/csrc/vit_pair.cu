@@ -8,10 +8,12 @@ namespace hmg {
 const void* vit_pair_ptr_g8(int q);
 const void* vit_pair_ptr_g16(int q);
 const void* vit_pair_ptr_g32(int q);
+const void* vit_pair_ptr_g32s(int q);
 
 int vit_pair_q_max() { return 16; }
 
-static const void* vit_pair_ptr(int G, int Q) {
+static const void* vit_pair_ptr(int G, int Q, bool scan) {
+  if (scan) return G == 32 ? vit_pair_ptr_g32s(Q) : nullptr;
   switch (G) {
     case 8: return vit_pair_ptr_g8(Q);
     case 16: return vit_pair_ptr_g16(Q);
@@ -20,8 +22,8 @@ static const void* vit_pair_ptr(int G, int Q) {
   return nullptr;
 }
 
-cudaError_t launch_vit_pair(int G, int Q, const VitArgs& a, cudaStream_t st, int* ok) {
-  const void* fn = vit_pair_ptr(G, Q);
+cudaError_t launch_vit_pair(int G, int Q, bool scan, const VitArgs& a, cudaStream_t st, int* ok) {
+  const void* fn = vit_pair_ptr(G, Q, scan);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
   const size_t smem = (((size_t)kRows * Q * G + 3) / 4) * 16;

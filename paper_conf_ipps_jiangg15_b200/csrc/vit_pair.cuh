@@ -35,9 +35,17 @@ namespace hmg {
 
 constexpr int kRedo = -65536;   // finish(): not a word score (those are >= -32768)
 
-template <int G, int Q>
+// SCAN: resolve the cross-lane D->D carries with one max-plus
+// prefix scan over the lanes (log2 G shuffle steps on (carry, tDD cost) pairs, both halves at
+// once, then the low -> high wrap) instead of vote-terminated passes.  A span of lanes maps an
+// incoming carry c to max(A, relu(c - C)) with C = -(sum of its tDD); spans compose as
+// (A1, C1) then (A2, C2) -> (max(A2, relu(A1 - C2)), C1 + C2).  Costs are kept as u16 clamped at
+// 32767 (exact: carries are <= 32767, so any larger cost yields the floor), added with one
+// VIADDMNMX.U16x2 min -- no wrap-around.  Same fixed point as the passes.
+template <int G, int Q, bool SCAN = false>
 struct VitPairLane {
   uint32_t tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q];   // s16x2 transitions
+  uint32_t bcost;            // SCAN: -(sum of the lane's tDD) per half, u16 clamped at 32767
   uint32_t Mc[Q], Ic[Q], Dc[Q], Bk[Q];                              // s16x2 cells (offset by F)
   uint32_t R;                // running max of M' over the rows
   uint32_t thrv;             // 0x8000 - threshold, per half: vote fires when R' >= threshold
@@ -56,6 +64,13 @@ struct VitPairLane {
       tII[q] = tr[6 * G * Q + o];
       tDD[q] = tr[7 * G * Q + o];
     }
+    int clo = 0, chi = 0;
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      clo = min(32767, clo - (int)(int16_t)(tDD[q] & 0xffffu));
+      chi = min(32767, chi - (int)(int16_t)(tDD[q] >> 16));
+    }
+    bcost = (uint32_t)clo | ((uint32_t)chi << 16);
   }
 
   // Bk' = sat16(xB + tBM_k) - F for both halves; false if a term exceeds the safe bound
@@ -186,6 +201,40 @@ struct VitPairLane {
       if (mine && bad) state = 2;
       if ((bal & gbits) && state) kill();
     }
+    if constexpr (SCAN) {
+      // inclusive max-plus scan of (carry out, tDD cost) over the lanes, both halves
+      uint32_t c = cout, sm = bcost;
+#pragma unroll
+      for (int d = 1; d < G; d <<= 1) {
+        const uint32_t c2 = __shfl_up_sync(0xffffffffu, c, d, G);
+        const uint32_t s2 = __shfl_up_sync(0xffffffffu, sm, d, G);
+        if (z >= d) {
+          c = __vimax_s16x2_relu(c, __vsub2(c2, sm));          // max(c, relu(c2 - cost))
+          sm = __viaddmin_u16x2(s2, sm, 0x7fff7fffu);           // cost sum, clamped
+        }
+      }
+      uint32_t cex = __shfl_up_sync(0xffffffffu, c, 1, G);
+      uint32_t sex = __shfl_up_sync(0xffffffffu, sm, 1, G);
+      const uint32_t wrap = __shfl_sync(0xffffffffu, c, G - 1, G) << 16;   // low chain out -> high
+      if (z == 0) cex = sex = 0u;
+      const uint32_t cin = __vimax_s16x2_relu(cex, __vsub2(wrap, sex));     // high: max(c, relu(wrap - C))
+      bool imp = __vmaxs2(cin, Dc[0]) != Dc[0];
+      if (__any_sync(0xffffffffu, imp)) {
+        Dc[0] = __vmaxs2(Dc[0], cin);
+        constexpr int K0 = Q < 3 ? Q : 3;
+#pragma unroll
+        for (int q = 1; q < K0; ++q) {
+          const uint32_t nd = __viaddmax_s16x2_relu(Dc[q - 1], tDD[q - 1], tDD[q - 1]);
+          imp = imp && (__vmaxs2(nd, Dc[q]) != Dc[q]);
+          Dc[q] = __vmaxs2(Dc[q], nd);
+        }
+        if (__any_sync(0xffffffffu, imp)) {
+#pragma unroll
+          for (int q = K0; q < Q; ++q) Dc[q] = __viaddmax_s16x2(Dc[q - 1], tDD[q - 1], Dc[q]);
+        }
+      }
+      return;
+    }
     // Lazy-F across virtual lanes (l.25, Fig 7): passes while any carry improves (reading R19)
     for (;;) {
       uint32_t cin = __shfl_sync(0xffffffffu, cout, src, G);
@@ -225,7 +274,7 @@ struct VitPairLane {
   }
 };
 
-template <int G, int Q>
+template <int G, int Q, bool SCAN = false>
 __global__ void __launch_bounds__(128) vit_pair_kernel(const VitArgs a) {
   constexpr int ROWW = Q * G;              // s16x2 words per residue row
   constexpr int NG = 32 / G;
@@ -243,7 +292,7 @@ __global__ void __launch_bounds__(128) vit_pair_kernel(const VitArgs a) {
   const int z = lane & (G - 1);
   const int grp = lane / G;
 
-  VitPairLane<G, Q> V;
+  VitPairLane<G, Q, SCAN> V;
   V.load(tr, z);
   const unsigned gbits = (G == 32 ? 0xffffffffu : ((1u << G) - 1u)) << (grp * G);
   const long long ntot = a.list ? *a.nlist : a.nseq;

@@ -544,3 +544,32 @@ def test_vit_block_pair_delete_chains_and_exits(W, monkeypatch):
         assert p.quant()["vit_pair_lanes"] >= 32 * W
         want = oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off)
         assert np.array_equal(got, want), M
+
+
+@pytest.mark.parametrize("M", [129, 300, 700, 1000])
+def test_vit_pair_maxplus_scan(M, monkeypatch):
+    """the cross-lane D->D carries of the pair kernel resolved by one max-plus
+    prefix scan (HMG_VIT_SCAN) instead of vote-terminated passes: identical raw scores on the
+    typical and the long-D-chain (Dir(1, 9)) profiles and on chains crossing every lane."""
+    monkeypatch.setenv("HMG_VIT_SCAN", "1")
+    rng = np.random.default_rng(M + 31)
+    for dd in [(7.0, 3.0), (1.0, 9.0)]:
+        prof = synth.make_profile(M, 600 + M, dd=dd)
+        dsq, off = _ragged_db(rng, n=40, alphabet=29, lmax=300)
+        got, p = _vit_gpu(prof.msc, prof.tsc, dsq, off)
+        assert p.quant()["vit_pair_lanes"] == 32
+        assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)), dd
+    msc = np.full((M, 29), -6.0, np.float32)
+    msc[0, 0] = 4.0
+    msc[M - 1, 1] = 4.0
+    tsc = np.log(rng.uniform(0.05, 1.0, size=(M, 8))).astype(np.float32)
+    tsc[:, 7] = np.log(rng.uniform(0.9, 0.9999, size=M))
+    tsc[:, 0] = np.log(1e-4 / M)
+    tsc[0, 0] = np.log(0.5)
+    tsc[0, 1:4] = -np.inf
+    tsc[M - 1, 4:8] = -np.inf
+    seqs = [np.array([0, 1], np.uint8), np.array([0, 2, 1], np.uint8)]
+    seqs += [synth.random_dsq(rng, int(L), 3) for L in rng.integers(1, 40, size=20)]
+    dsq, off = _db_from(seqs)
+    got, _ = _vit_gpu(msc, tsc, dsq, off)
+    assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
