@@ -16,6 +16,8 @@ Parity status per function:
   Viterbi DP ..................... pinned (brute-force Plan-7 paths, wide-int
                                    recompute, ungapped special case)
   nats / null1 / Gumbel / pass ... pinned (closed forms, textbook Gumbel)
+  Forward score (f2) ............. pinned (brute-force sum over all Plan-7 paths with
+                                   N/J/C loops, closed form for a one-node model)
   agreement with HMMER 3.0 itself  parity unpinned (no HMMER source or scores
                                    on this box; R1-R34)
 """
@@ -67,6 +69,8 @@ def lib():
             "or_msv_pass": (c_int, [c_int, c_int, c_double, c_double, c_double]),
             "or_vit_pass": (c_int, [c_int, c_int, c_double, c_double, c_double]),
             "or_bits": (c_double, [c_float, c_int]),
+            "or_fwd_seq": (c_double, [c_int, c_p, c_p, c_p, c_int, c_p]),
+            "or_fwd_db": (None, [c_int, c_p, c_p, c_p, c_p, c_p, c_i64, c_int, c_p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -157,6 +161,33 @@ def vit_db(p: VitProfile, dsq: np.ndarray, off: np.ndarray, ids=None, nthreads: 
         idp = _ptr(ids)
     out = np.zeros(n, dtype=np.int32)
     lib().or_vit_db(p.M, _ptr(p.rsc), _ptr(p.tr), _ptr(dsq), _ptr(off), idp, n,
+                    nthreads or os.cpu_count() or 1, _ptr(out))
+    return out
+
+
+def fwd_seq(msc: np.ndarray, tsc: np.ndarray, dsq: np.ndarray) -> float:
+    """Forward score in nats ("total log-likelihood ratios summed over
+    all possible alignments", Fig 1), double precision log space."""
+    msc = np.ascontiguousarray(msc, dtype=np.float32)
+    tsc = np.ascontiguousarray(tsc, dtype=np.float32)
+    d = np.ascontiguousarray(dsq, dtype=np.uint8)
+    M = msc.shape[0]
+    scratch = np.zeros(6 * (M + 1), dtype=np.float64)
+    return lib().or_fwd_seq(M, _ptr(msc), _ptr(tsc), _ptr(d), len(d), _ptr(scratch))
+
+
+def fwd_db(msc, tsc, dsq, off, ids=None, nthreads: int | None = None) -> np.ndarray:
+    msc = np.ascontiguousarray(msc, dtype=np.float32)
+    tsc = np.ascontiguousarray(tsc, dtype=np.float32)
+    dsq = np.ascontiguousarray(dsq, dtype=np.uint8)
+    off = np.ascontiguousarray(off, dtype=np.int64)
+    n = len(off) - 1 if ids is None else len(ids)
+    idp = None
+    if ids is not None:
+        ids = np.ascontiguousarray(ids, dtype=np.int64)
+        idp = _ptr(ids)
+    out = np.zeros(n, dtype=np.float64)
+    lib().or_fwd_db(msc.shape[0], _ptr(msc), _ptr(tsc), _ptr(dsq), _ptr(off), idp, n,
                     nthreads or os.cpu_count() or 1, _ptr(out))
     return out
 

@@ -22,7 +22,12 @@
  *      every row (Lazy-F, P:519-533 / P:727-790, is an exact shortcut of this
  *      closure, so the oracle does not take it);
  *   4. score conversion to nats, null1, Gumbel survival and pass decisions
- *      (HMMER 3.0 pipeline reading, R9-R12).
+ *      (HMMER 3.0 pipeline reading, R9-R12);
+ *   5. Forward score: "the total log-likelihood ratios summed
+ *      over all possible alignments" of the same Plan-7 local
+ *      multihit model (Fig 3), in double precision log space, the textbook
+ *      Forward recurrence with HMMER 3.0's full length model (readings F1-F5 in
+ *      DESIGN.md); the stage after P7Viterbi in Fig 1.
  *
  * Layouts (same meaning as include/hmg.h, restated, not shared):
  *   msc : float32 [M][29] log-odds in nats, residue order
@@ -363,3 +368,96 @@ int or_vit_pass(int raw, int L, double mu, double lambda, double F) {
 
 /* Bits score (for mu calibration): (nats - null1)/ln2. */
 double or_bits(float nats, int L) { return (double)(nats - or_null1(L)) / OR_LN2; }
+
+/* ------------------------------------------------------------------------ */
+/* 5. Forward score (f2; "summed over all possible alignments",      */
+/*    Fig 1; readings F1-F5)                                       */
+/* ------------------------------------------------------------------------ */
+
+static double or_lse(double a, double b) {            /* log(e^a + e^b), -inf aware */
+  if (a == -INFINITY) return b;
+  if (b == -INFINITY) return a;
+  return a > b ? a + log1p(exp(b - a)) : b + log1p(exp(a - b));
+}
+
+/* Forward score in nats of one sequence: log of the summed odds of every path
+ * S -> N* -> B -> (M|I|D)+ -> E -> (J -> B ...)* -> C* -> T, where
+ *   emissions: M_k emits x with odds exp(msc[k][x]); I_k, N, C, J emit with odds 1 (F3, F4);
+ *   transitions: the profile's tsc (log probabilities; -inf = absent), local entry
+ *   B->M_k = tsc[k][BM], local exit M_k->E and D_k->E = 1 (F1), E->C = E->J = 1/2 (R9),
+ *   length model N->N = J->J = C->C = L/(L+3), N->B = J->B = C->T = 3/(L+3) (F2).
+ * Rows are computed in the paper's order (Alg 2's row loop, with sums in place of
+ * maxima): M and I from row i-1, D along row i, then E, N, J, C, B (F5). */
+double or_fwd_seq(int M, const float* msc, const float* tsc, const uint8_t* dsq, int L, double* scratch) {
+  double* Mp = scratch;            double* Ip = Mp + (M + 1);   double* Dp = Ip + (M + 1);
+  double* Mn = Dp + (M + 1);       double* In = Mn + (M + 1);   double* Dn = In + (M + 1);
+  const double loop = log((double)L / (double)(L + 3)), move = log(3.0 / (double)(L + 3));
+  const double half = log(0.5);
+#define TS(k, t) ((double)tsc[(size_t)((k) - 1) * 8 + (t)])   /* node k = 1..M */
+  for (int k = 0; k <= M; ++k) Mp[k] = Ip[k] = Dp[k] = -INFINITY;
+  double N = 0.0, J = -INFINITY, C = -INFINITY, B = N + move;     /* row 0 */
+  for (int i = 0; i < L; ++i) {
+    const int x = dsq[i];
+    Mn[0] = In[0] = Dn[0] = -INFINITY;
+    for (int k = 1; k <= M; ++k) {
+      double sm = B + TS(k, 0);                                      /* B -> M_k */
+      if (k > 1) {
+        sm = or_lse(sm, Mp[k - 1] + TS(k, 1));                       /* M_{k-1} -> M_k */
+        sm = or_lse(sm, Ip[k - 1] + TS(k, 2));                       /* I_{k-1} -> M_k */
+        sm = or_lse(sm, Dp[k - 1] + TS(k, 3));                       /* D_{k-1} -> M_k */
+      }
+      Mn[k] = sm + (double)msc[(size_t)(k - 1) * OR_K + x];
+      In[k] = (k < M) ? or_lse(Mp[k] + TS(k, 5), Ip[k] + TS(k, 6)) : -INFINITY;   /* odds 1 */
+      Dn[k] = (k > 1) ? or_lse(Mn[k - 1] + TS(k - 1, 4), Dn[k - 1] + TS(k - 1, 7)) : -INFINITY;
+    }
+    double E = -INFINITY;
+    for (int k = 1; k <= M; ++k) E = or_lse(E, or_lse(Mn[k], Dn[k]));     /* M_k, D_k -> E */
+    N = N + loop;
+    J = or_lse(J + loop, E + half);
+    C = or_lse(C + loop, E + half);
+    B = or_lse(N + move, J + move);
+    double* t;
+    t = Mp; Mp = Mn; Mn = t;
+    t = Ip; Ip = In; In = t;
+    t = Dp; Dp = Dn; Dn = t;
+  }
+#undef TS
+  return C + move;                                                    /* C -> T */
+}
+
+typedef struct {
+  int M; const float* msc; const float* tsc;
+  const uint8_t* dsq; const int64_t* off; const int64_t* ids; int64_t n;
+  double* out; int64_t next; pthread_mutex_t mu;
+} or_fjob;
+
+static void* or_fworker(void* arg) {
+  or_fjob* J = (or_fjob*)arg;
+  double* scratch = (double*)malloc(sizeof(double) * 6 * (size_t)(J->M + 1));
+  for (;;) {
+    int64_t lo, hi;
+    pthread_mutex_lock(&J->mu);
+    lo = J->next; hi = lo + 4; if (hi > J->n) hi = J->n; J->next = hi;
+    pthread_mutex_unlock(&J->mu);
+    if (lo >= J->n) break;
+    for (int64_t j = lo; j < hi; ++j) {
+      int64_t s = J->ids ? J->ids[j] : j;
+      J->out[j] = or_fwd_seq(J->M, J->msc, J->tsc, J->dsq + J->off[s], (int)(J->off[s + 1] - J->off[s]), scratch);
+    }
+  }
+  free(scratch);
+  return 0;
+}
+
+void or_fwd_db(int M, const float* msc, const float* tsc, const uint8_t* dsq, const int64_t* off,
+               const int64_t* ids, int64_t n, int nthreads, double* out) {
+  or_fjob J; memset(&J, 0, sizeof J);
+  J.M = M; J.msc = msc; J.tsc = tsc; J.dsq = dsq; J.off = off; J.ids = ids; J.n = n; J.out = out;
+  if (nthreads < 1) nthreads = 1;
+  pthread_mutex_init(&J.mu, 0);
+  pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * (size_t)nthreads);
+  for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], 0, or_fworker, &J);
+  for (int t = 0; t < nthreads; ++t) pthread_join(th[t], 0);
+  free(th);
+  pthread_mutex_destroy(&J.mu);
+}

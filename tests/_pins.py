@@ -15,6 +15,9 @@ by a route different from the oracle's row-by-row DP:
   nothing improves -- it must equal the full closure the oracle performs.
 * ``vit_ungapped``: the Viterbi filter with no I and no D states written as its
   own 20-line DP.
+* ``fwd_brute``: the Forward score ("summed over all possible
+  alignments") as an explicit sum over every state path of the Plan-7
+  multihit model with its N/J/C length model, in float64 (fsum of exp).
 """
 from __future__ import annotations
 
@@ -243,3 +246,66 @@ def vit_ungapped(rsc, tbm, tmm, move, dsq, xw_e=-500):
         xB = max(xJ, 12000) + move
         prev = cur
     return xC
+
+
+def fwd_brute(msc, tsc, dsq, stats=False):
+    """log of the sum over ALL state paths S->N->B->(M|I|D)->E->(J->B..)->C->T of the path's
+    odds (emission odds exp(msc) for M, 1 for I/N/J/C; transition probabilities exp(tsc);
+    local entry B->M_k, local exit M_k->E and D_k->E with probability 1, E->C = E->J = 1/2,
+    N->N = J->J = C->C = L/(L+3), N->B = J->B = C->T = 3/(L+3)).  Depth-first enumeration,
+    tiny M and L only."""
+    import math
+    M, L = msc.shape[0], len(dsq)
+    loop, move = math.log(L / (L + 3.0)), math.log(3.0 / (L + 3.0))
+    half = math.log(0.5)
+    T = lambda k, t: float(tsc[k - 1, t])       # node k = 1..M
+    terms = []
+    sys.setrecursionlimit(10000)
+
+    def go(state, k, i, v):                      # i residues emitted so far, v log-odds so far
+        if v == -math.inf:
+            return
+        if state == "N":
+            if i < L:
+                go("N", 0, i + 1, v + loop)      # N loop emits residue i+1
+            go("B", 0, i, v + move)
+        elif state == "B":
+            if i < L:
+                for kk in range(1, M + 1):
+                    go("M", kk, i + 1, v + T(kk, 0) + float(msc[kk - 1, dsq[i]]))
+        elif state == "M":
+            go("E", 0, i, v)                     # local exit
+            if k < M:
+                if i < L:
+                    go("M", k + 1, i + 1, v + T(k + 1, 1) + float(msc[k, dsq[i]]))
+                    go("I", k, i + 1, v + T(k, 5))
+                go("D", k + 1, i, v + T(k, 4))
+        elif state == "I":
+            if i < L:
+                go("M", k + 1, i + 1, v + T(k + 1, 2) + float(msc[k, dsq[i]]))
+                go("I", k, i + 1, v + T(k, 6))
+        elif state == "D":
+            go("E", 0, i, v)                     # local exit
+            if k < M:
+                if i < L:
+                    go("M", k + 1, i + 1, v + T(k + 1, 3) + float(msc[k, dsq[i]]))
+                go("D", k + 1, i, v + T(k, 7))
+        elif state == "E":
+            go("C", 0, i, v + half)
+            go("J", 0, i, v + half)
+        elif state == "J":
+            if i < L:
+                go("J", 0, i + 1, v + loop)
+            go("B", 0, i, v + move)
+        elif state == "C":
+            if i < L:
+                go("C", 0, i + 1, v + loop)
+            else:
+                terms.append(v + move)           # C -> T after the last residue
+
+    go("N", 0, 0, 0.0)
+    if not terms:
+        return (-math.inf, -math.inf, 0) if stats else -math.inf
+    top = max(terms)
+    lse = top + math.log(math.fsum(math.exp(t - top) for t in terms))
+    return (lse, top, len(terms)) if stats else lse

@@ -373,3 +373,49 @@ def test_vit_long_delete_chain(seed):
         move = oracle.move_w(L)
         want = _pins.vit_wide(p.rsc, p.tr, move, dsq)
         assert oracle.vit_seq(p, dsq) == want == _pins.vit_lazyf(p.rsc, p.tr, move, p.ddbound, dsq)
+
+
+# ------------------------------------------------------------------ Forward (f2)
+@pytest.mark.parametrize("seed", range(6))
+def test_fwd_brute_force(seed):
+    """Forward = log of the sum over every Plan-7 path, enumerated explicitly; includes
+    I self-loops, D chains with D->E exits, multihit J and the N/C loops."""
+    rng = np.random.default_rng(400 + seed)
+    M = int(rng.integers(1, 4))
+    msc = rng.uniform(-3.0, 2.5, size=(M, 29)).astype(np.float32)
+    msc[:, 20] = -np.inf
+    tsc = np.log(rng.uniform(0.05, 0.9, size=(M, 8))).astype(np.float32)
+    tsc[0, 1:4] = -np.inf
+    tsc[M - 1, 4:8] = -np.inf
+    for L in (1, 2, 3, 4):
+        d = rng.integers(0, 20, size=L).astype(np.uint8)
+        want = _pins.fwd_brute(msc, tsc, d)
+        got = oracle.fwd_seq(msc, tsc, d)
+        assert got == pytest.approx(want, rel=1e-12, abs=1e-12), (M, L)
+
+
+def test_fwd_closed_form_one_node():
+    """M = 1, L = 1: the only path is N->B->M_1->E->C->T, so
+    fwd = 2 log(3/4) + tBM + msc[x] + log(1/2)."""
+    msc = np.full((1, 29), -1.0, np.float32)
+    msc[0, 7] = 1.25
+    tsc = np.full((1, 8), -np.inf, np.float32)
+    tsc[0, 0] = np.log(0.3)
+    got = oracle.fwd_seq(msc, tsc, np.array([7], np.uint8))
+    want = 2 * math.log(0.75) + float(np.float32(np.log(0.3))) + 1.25 + math.log(0.5)
+    assert got == pytest.approx(want, rel=1e-12)
+
+
+def test_fwd_bounds_best_path():
+    """A sum of path odds lies between its largest term (the unquantised Viterbi path) and that
+    term times the number of paths; the oracle's DP must respect both bounds."""
+    rng = np.random.default_rng(9)
+    for M in (1, 2, 3):
+        msc = rng.uniform(-2.0, 2.0, size=(M, 29)).astype(np.float32)
+        tsc = np.log(rng.uniform(0.1, 0.9, size=(M, 8))).astype(np.float32)
+        tsc[0, 1:4] = -np.inf
+        tsc[M - 1, 4:8] = -np.inf
+        d = rng.integers(0, 20, size=4).astype(np.uint8)
+        _, best, npath = _pins.fwd_brute(msc, tsc, d, stats=True)
+        f = oracle.fwd_seq(msc, tsc, d)
+        assert best - 1e-12 <= f <= best + math.log(npath) + 1e-12
