@@ -75,6 +75,9 @@ typedef struct {
   int vit_pair_lanes, vit_pair_regs; /* s16x2 pair Viterbi kernel (two cells per register) in front of
                                         the s32 kernel: lanes per sequence G, s16x2 registers Q per
                                         cell type; 0 = not used for this profile */
+  int fwd_warps, fwd_nodes;         /* Forward kernel geometry: warps per sequence W, nodes per thread Q
+                                       (0 = no Forward stage: no tsc, or M > 4096) */
+  int fwd_rows_smem;                /* emission-odds rows staged in shared memory (the rest via L1) */
 } hmg_quant;
 
 /* ---------------------------------------------------------------- profile */
@@ -179,17 +182,43 @@ hmg_status hmg_pipeline(const hmg_profile* p, const hmg_db* db, double F1, doubl
                         uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
                         int64_t* n_survivors);
 
+/* Forward stage (Fig 1, the filter after P7Viterbi; "total
+ * log-likelihood ratios summed over all possible alignments") over the n sequences
+ * listed in `ids` (device int32, caller order; NULL = all sequences, n ignored).
+ * Model: the same Plan-7 local multihit profile, in float32 odds space (emission odds
+ * exp(msc), transition odds exp(tsc), exits M_k/D_k -> E = 1, E -> J = E -> C = 1/2, length
+ * model N->N = J->J = C->C = L/(L+3), N->B = J->B = C->T = 3/(L+3); readings F1-F5),
+ * rows rescaled by exact powers of two.
+ *   nats : device float32 [nseq], written at the listed indices: the Forward score in nats
+ *          (log of the summed path odds; -INFINITY if no path has non-zero odds).
+ * Accuracy: float32 rounding, |error| <= 2^-24 (40 L + 4 M) + 1e-6 nats against exact arithmetic
+ * on the paths that carry the score.  Needs tsc; HMG_EUNSUPPORTED for M > 4096
+ * or emission log-odds above +40 nats (odds-space range). */
+hmg_status hmg_forward(const hmg_profile* p, const hmg_db* db, const int32_t* ids, int64_t n, void* stream,
+                       float* nats);
+
+/* hmg_pipeline followed by the Forward stage on the sequences that passed the Viterbi filter
+ * (Fig 1: MSV -> P7Viterbi -> Forward).  Outputs of hmg_pipeline, plus:
+ *   fwd_nats  float32 [nseq]  Forward score (nats) of the Viterbi passes, written at those only
+ *   fwd_ids   int32 [nseq]    caller indices of the Viterbi passes, length-descending order
+ *   n_fwd     int64 [1]       device count of fwd_ids
+ * and flags bit3 = the Forward stage ran for this sequence. */
+hmg_status hmg_pipeline_forward(const hmg_profile* p, const hmg_db* db, double F1, double F2, void* stream,
+                                uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                                int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids, int64_t* n_fwd);
+
 /* ---------------------------------------------------------------- instrumentation */
 
 /* Number of CUDA kernels this library has launched since it was loaded. */
 int64_t hmg_kernel_launches(void);
 
 /* Stage timing (profiling aid, off by default).  When enabled, hmg_msv /
- * hmg_viterbi / hmg_pipeline record CUDA events on their stream between
- * stages; hmg_stage_times waits for the last recorded event and fills
- * ms[5] with the durations of the most recent call's stages (-1 = not run):
+ * hmg_viterbi / hmg_pipeline / hmg_forward / hmg_pipeline_forward record CUDA events on their
+ * stream between stages; hmg_stage_times waits for the last recorded event and fills
+ * ms[6] with the durations of the most recent call's stages (-1 = not run):
  *   0 MSV fast kernel   1 MSV exact re-scoring (select + kernel)
  *   2 MSV pass flags + survivor compaction   3 Viterbi kernel   4 Viterbi flags/scatter
+ *   5 Viterbi-pass compaction + Forward kernel
  * Not thread-safe across concurrent calls (one global set of events). */
 hmg_status hmg_set_stage_timing(int enable);
 hmg_status hmg_stage_times(double* ms);

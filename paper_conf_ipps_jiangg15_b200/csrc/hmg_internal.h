@@ -79,6 +79,23 @@ struct LongArgs {
   unsigned long long* counter;  // [2] work queues (chunks, Viterbi)
 };
 
+// Forward filter stage (forward.cu): float odds-space Forward over a sorted list
+struct FwdArgs {
+  const uint32_t* words;
+  const uint32_t* woff16;
+  const int32_t* len;
+  const int32_t* order;        // sorted -> caller
+  const int32_t* list;         // sorted indices (NULL = all)
+  const int64_t* nlist;        // device count when list != NULL
+  int64_t nseq;
+  const float* etab;           // [kRows][C][T][V] emission odds (chunked), full copy in global memory
+  const float* tr;             // [8][T][Q] transition odds
+  int rows_smem;               // residue rows staged in shared memory (x < rows_smem)
+  float* out;                  // [nseq] caller order, nats
+  uint8_t* flags;              // [nseq] caller order or NULL: bit 3 set when the Forward stage ran
+  unsigned long long* counter;
+};
+
 }  // namespace hmg
 
 struct hmg_profile {
@@ -114,6 +131,11 @@ struct hmg_profile {
   uint32_t* d_long_msv = nullptr;
   int32_t* d_long_rsc = nullptr;
   int32_t* d_long_tr = nullptr;
+  // Forward stage (forward.cu): fwd_kernel<fwd_W, fwd_Q>, emission rows x < fwd_rows in shared memory
+  int fwd_W = 0, fwd_Q = 0, fwd_rows = 0;
+  float msc_max = 0.f;              // largest emission log-odds (odds-space range check)
+  float* d_fwd_e = nullptr;         // emission odds [kRows][C][T][V]
+  float* d_fwd_t = nullptr;         // transition odds [8][T][Q]
   // threshold caches (built on first use per F and DB Lmax)
   std::mutex mu;
   struct Thr {
@@ -175,7 +197,16 @@ cudaError_t msv_finish(const uint8_t* raw_sorted, const int32_t* len, const int3
                        int64_t* nsurv, int32_t* surv_caller, void* tmp, cudaStream_t st);
 cudaError_t vit_finish(const int16_t* raw_sorted, const int32_t* list, const int64_t* nlist, int64_t nmax,
                        const int32_t* len, const int32_t* order, const int32_t* thr, int16_t* raw_out,
-                       uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st);
+                       uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st, uint8_t* pass_sorted = nullptr);
+cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* order, int32_t* ids_sorted,
+                          int32_t* ids_caller, int64_t* count, void* tmp, cudaStream_t st);
+
+// Forward stage (forward.cu)
+bool fwd_geometry(int M, int* W, int* Q);
+size_t fwd_smem(int W, int Q, int rows);
+void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
+                std::vector<float>* tr);
+cudaError_t launch_fwd(int W, int Q, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok);
 cudaError_t to_sorted_ids(const int32_t* caller_ids, int64_t n, const int32_t* inv_order, int32_t* sorted_ids,
                           cudaStream_t st);
 cudaError_t set_count(int64_t* d, int64_t v, cudaStream_t st);

@@ -27,8 +27,8 @@ namespace {
 
 // ---------------------------------------------------------------- stage timing (profiling aid)
 // Stages: 0 MSV fast kernel | 1 MSV exact redo (select + kernel) | 2 MSV flags + compaction |
-//         3 Viterbi kernel | 4 Viterbi flags/scatter.  Marks are CUDA events on the call's stream.
-constexpr int kStages = 5;
+//         3 Viterbi kernel | 4 Viterbi flags/scatter | 5 Viterbi-pass compaction + Forward kernel.  Marks are CUDA events on the call's stream.
+constexpr int kStages = 6;
 struct StageTimer {
   bool on = false;
   int device = -1;
@@ -55,6 +55,7 @@ void stage_count_redo(const unsigned long long* d, cudaStream_t st) {
 }
 
 constexpr double kLn2 = 0.693147180559945309417232121458176568;
+constexpr float kFwdMscMax = 40.0f;   // Forward odds space: emission log-odds above this could overflow float
 
 // ---------------------------------------------------------------- quantisation
 struct Scales {
@@ -775,6 +776,17 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     p->has_ev = true;
     p->ev = *ev;
   }
+  p->msc_max = -INFINITY;
+  for (size_t i = 0; i < (size_t)M * kAlpha; ++i) p->msc_max = std::max(p->msc_max, msc[i]);
+  // ---- Forward stage geometry (forward.cu): emission rows staged in shared memory as fit
+  if (tsc && fwd_geometry(M, &p->fwd_W, &p->fwd_Q)) {
+    int smax = 0;
+    if (device >= 0) cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+    else smax = 227 * 1024;
+    int rows = kAlpha;
+    while (rows > 0 && fwd_smem(p->fwd_W, p->fwd_Q, rows) > (size_t)smax) --rows;
+    p->fwd_rows = rows;
+  }
   // ---- kernel geometry and device tables
   p->msv_fast = p->bias < 66 + p->tbm;   // precondition of the fast MSV kernel
   msv_geometry(M, &p->msv_G, &p->msv_Q);
@@ -932,6 +944,12 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       }
     }
   }
+  if (st == HMG_OK && p->fwd_W > 0) {
+    std::vector<float> e, t;
+    fwd_tables(M, p->fwd_W, p->fwd_Q, msc, tsc, &e, &t);
+    st = upload(&p->d_fwd_e, e.data(), e.size());
+    if (st == HMG_OK) st = upload(&p->d_fwd_t, t.data(), t.size());
+  }
   if (st != HMG_OK) {
     hmg_profile_destroy(p);
     return st;
@@ -1025,6 +1043,9 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->vit_nodes = p->vit_generic ? 0 : p->vit_Q;
   q->vit_pair_lanes = p->pair_G;
   q->vit_pair_regs = p->pair_Q;
+  q->fwd_warps = p->fwd_W;
+  q->fwd_nodes = p->fwd_Q;
+  q->fwd_rows_smem = p->fwd_rows;
   return HMG_OK;
 }
 
@@ -1041,6 +1062,8 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_long_tr);
     cudaFree(p->d_pair_rsc);
     cudaFree(p->d_pair_tr);
+    cudaFree(p->d_fwd_e);
+    cudaFree(p->d_fwd_t);
     cudaFree(p->thr_msv.d);
     cudaFree(p->thr_vit.d);
     cudaGetLastError();
@@ -1283,9 +1306,9 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
   return cuda_status(e);
 }
 
-hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
-                        uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
-                        int64_t* n_survivors) {
+static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
+                                uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                                int64_t* n_survivors, uint8_t* vpass_sorted) {
   hmg_profile* p = const_cast<hmg_profile*>(pc);
   if (!p || !db || !p->has_tsc || !p->has_ev || p->device != db->device || db->device < 0) return HMG_EINVAL;
   if (!(F1 > 0.0 && F1 <= 1.0) || !(F2 > 0.0 && F2 <= 1.0)) return HMG_EINVAL;
@@ -1352,11 +1375,110 @@ hmg_status hmg_pipeline(const hmg_profile* pc, const hmg_db* db, double F1, doub
     s = run_vit(p, db, surv, n_survivors, st, vraw_sorted, S, owned, nlong);  // P7Viterbi on survivors
     if (s != HMG_OK) return s;
 
-    e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st);
+    e = vit_finish(vraw_sorted, surv, n_survivors, n, db->d_len, db->d_order, tv, vit_raw, nullptr, flags, st,
+                   vpass_sorted);
     mark(5, st);
   }
   if (e == cudaSuccess) e = cudaGetLastError();
   return cuda_status(e);
 }
 
+
+hmg_status hmg_pipeline(const hmg_profile* p, const hmg_db* db, double F1, double F2, void* stream,
+                        uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                        int64_t* n_survivors) {
+  return pipeline_impl(p, db, F1, F2, stream, msv_raw, vit_raw, flags, survivor_ids, n_survivors, nullptr);
+}
+
+// Forward stage over a sorted-order list (device list + device count, nmax = list capacity).
+static hmg_status run_fwd(const hmg_profile* p, const hmg_db* db, const int32_t* list, const int64_t* nlist,
+                          cudaStream_t st, float* nats, uint8_t* flags, Scratch& S) {
+  if (p->fwd_W == 0) return HMG_EUNSUPPORTED;
+  cudaError_t e = cudaSuccess;
+  auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long), &e);
+  if (e) return cuda_status(e);
+  if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long), st))) return cuda_status(e);
+  FwdArgs a{};
+  a.words = db->d_words;
+  a.woff16 = db->d_woff16;
+  a.len = db->d_len;
+  a.order = db->d_order;
+  a.list = list;
+  a.nlist = nlist;
+  a.nseq = db->nseq;
+  a.etab = p->d_fwd_e;
+  a.tr = p->d_fwd_t;
+  a.rows_smem = p->fwd_rows;
+  a.out = nats;
+  a.flags = flags;
+  a.counter = ctr;
+  int ok = 0;
+  if ((e = launch_fwd(p->fwd_W, p->fwd_Q, p->fwd_rows, a, st, &ok))) return cuda_status(e);
+  return ok ? HMG_OK : HMG_EUNSUPPORTED;
+}
+
+hmg_status hmg_forward(const hmg_profile* pc, const hmg_db* db, const int32_t* ids, int64_t n, void* stream,
+                       float* nats) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !db || !p->has_tsc || (!nats && db->nseq) || p->device != db->device || db->device < 0)
+    return HMG_EINVAL;
+  if (ids && n < 0) return HMG_EINVAL;
+  if (p->fwd_W == 0 || p->msc_max > kFwdMscMax) return HMG_EUNSUPPORTED;
+  if (db->nseq == 0 || (ids && n == 0)) return HMG_OK;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = cudaSuccess;
+  hmg_status s;
+  {
+    Scratch S(st);
+    const int32_t* list = nullptr;
+    const int64_t* nl = nullptr;
+    if (ids) {
+      auto* sl = (int32_t*)S.get(sizeof(int32_t) * (size_t)n, &e);
+      auto* cnt = (int64_t*)S.get(sizeof(int64_t), &e);
+      if (e) return cuda_status(e);
+      if ((e = to_sorted_ids(ids, n, db->d_inv, sl, st))) return cuda_status(e);
+      if ((e = set_count(cnt, n, st))) return cuda_status(e);
+      list = sl;
+      nl = cnt;
+    }
+    mark_reset();
+    mark(5, st);
+    s = run_fwd(p, db, list, nl, st, nats, nullptr, S);
+    mark(6, st);
+  }
+  if (s != HMG_OK) return s;
+  return cuda_status(cudaGetLastError());
+}
+
+hmg_status hmg_pipeline_forward(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
+                                uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
+                                int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids, int64_t* n_fwd) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !db || p->device != db->device || db->device < 0) return HMG_EINVAL;
+  if (db->nseq && (!fwd_nats || !fwd_ids || !n_fwd)) return HMG_EINVAL;
+  if (p->has_tsc && (p->fwd_W == 0 || p->msc_max > kFwdMscMax)) return HMG_EUNSUPPORTED;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t n = db->nseq;
+  cudaError_t e = cudaSuccess;
+  hmg_status s;
+  {
+    Scratch S(st);
+    auto* vpass = (uint8_t*)S.get((size_t)std::max<int64_t>(n, 1), &e);
+    auto* fl = (int32_t*)S.get(sizeof(int32_t) * (size_t)std::max<int64_t>(n, 1), &e);
+    void* tmp = S.get(scan_tmp_bytes(n) + 16, &e);
+    if (e) return cuda_status(e);
+    if (n && (e = cudaMemsetAsync(vpass, 0, (size_t)n, st))) return cuda_status(e);
+    s = pipeline_impl(p, db, F1, F2, stream, msv_raw, vit_raw, flags, survivor_ids, n_survivors, vpass);
+    if (s != HMG_OK) return s;
+    if (n == 0) return n_fwd ? cuda_status(set_count(n_fwd, 0, st)) : HMG_OK;
+    // Viterbi passes -> Forward list (stable, schedule order) -> Forward kernel (Fig 1)
+    if ((e = compact_flags(vpass, n, db->d_order, fl, fwd_ids, n_fwd, tmp, st))) return cuda_status(e);
+    s = run_fwd(p, db, fl, n_fwd, st, fwd_nats, flags, S);
+    mark(6, st);
+  }
+  if (s != HMG_OK) return s;
+  return cuda_status(cudaGetLastError());
+}
 }  // extern "C"

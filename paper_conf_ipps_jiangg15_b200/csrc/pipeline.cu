@@ -116,6 +116,12 @@ static cudaError_t compact(const uint8_t* flag, int64_t n, const int32_t* order,
   return cudaGetLastError();
 }
 
+// stable compaction of a sorted-order flag array (Viterbi passes -> Forward list)
+cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* order, int32_t* ids_sorted,
+                          int32_t* ids_caller, int64_t* count, void* tmp, cudaStream_t st) {
+  return compact(flag_sorted, n, order, ids_sorted, ids_caller, count, tmp, st);
+}
+
 __global__ void redo_flag_kernel(const uint8_t* __restrict__ raw, int64_t n, uint8_t* __restrict__ flag) {
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
     flag[k] = raw[k] == 254;
@@ -165,7 +171,7 @@ __global__ void vit_flag_kernel(const int16_t* __restrict__ raw, const int32_t* 
                                 const int64_t* __restrict__ nlist, int64_t nmax, const int32_t* __restrict__ len,
                                 const int32_t* __restrict__ order, const int32_t* __restrict__ thr,
                                 int16_t* __restrict__ raw_out, uint8_t* __restrict__ pass_out,
-                                uint8_t* __restrict__ flags_out) {
+                                uint8_t* __restrict__ flags_out, uint8_t* __restrict__ pass_sorted) {
   const int64_t n = list ? *nlist : nmax;
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
     const int s = list ? list[j] : (int)j;
@@ -175,17 +181,18 @@ __global__ void vit_flag_kernel(const int16_t* __restrict__ raw, const int32_t* 
     const bool p = thr ? (r == 32767 || r >= thr[len[s]]) : false;
     if (pass_out) pass_out[c] = p;
     if (flags_out) flags_out[c] = (uint8_t)(flags_out[c] | 4u | (p ? 2u : 0u));
+    if (pass_sorted) pass_sorted[s] = p;
   }
 }
 
 cudaError_t vit_finish(const int16_t* raw_sorted, const int32_t* list, const int64_t* nlist, int64_t nmax,
                        const int32_t* len, const int32_t* order, const int32_t* thr, int16_t* raw_out,
-                       uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st) {
+                       uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st, uint8_t* pass_sorted) {
   if (nmax <= 0) return cudaSuccess;
   const int64_t b = (nmax + 255) / 256;
   g_launches += 1;
   vit_flag_kernel<<<(unsigned)(b < 8192 ? b : 8192), 256, 0, st>>>(raw_sorted, list, nlist, nmax, len, order, thr,
-                                                                    raw_out, pass_out, flags_out);
+                                                                    raw_out, pass_out, flags_out, pass_sorted);
   return cudaGetLastError();
 }
 

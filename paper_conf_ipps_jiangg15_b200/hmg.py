@@ -31,7 +31,8 @@ class hmg_quant(ctypes.Structure):
                 ("cost", ctypes.POINTER(ctypes.c_uint8)), ("rsc", ctypes.POINTER(ctypes.c_int16)),
                 ("tsc", ctypes.POINTER(ctypes.c_int16)), ("msv_fast", c_int), ("msv_lanes", c_int),
                 ("msv_regs", c_int), ("vit_lanes", c_int), ("vit_nodes", c_int),
-                ("vit_pair_lanes", c_int), ("vit_pair_regs", c_int)]
+                ("vit_pair_lanes", c_int), ("vit_pair_regs", c_int),
+                ("fwd_warps", c_int), ("fwd_nodes", c_int), ("fwd_rows_smem", c_int)]
 
 
 # name -> (restype, argtypes), exactly the declarations of include/hmg.h
@@ -51,6 +52,8 @@ SIGNATURES = {
     "hmg_msv": (c_int, [c_p, c_p, c_d, c_p, c_p, c_p]),
     "hmg_viterbi": (c_int, [c_p, c_p, c_p, c_i64, c_d, c_p, c_p, c_p]),
     "hmg_pipeline": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
+    "hmg_forward": (c_int, [c_p, c_p, c_p, c_i64, c_p, c_p]),
+    "hmg_pipeline_forward": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_nats": (c_f, [c_int, c_int]),
     "hmg_vit_nats": (c_f, [c_int, c_int]),
     "hmg_null1_nats": (c_f, [c_int]),
@@ -249,6 +252,23 @@ def hmg_pipeline(profile: Profile, db: Database, msv_raw, vit_raw, flags, surviv
                               _dev_ptr(n_survivors)), "hmg_pipeline")
 
 
+def hmg_forward(profile: Profile, db: Database, nats, ids=None, stream=None):
+    """Forward stage (f2; Fig 1) over device int32 ``ids`` (caller order; None = all)
+    into the device float32 tensor ``nats`` [nseq]."""
+    n = 0 if ids is None else int(ids.numel())
+    _check(lib().hmg_forward(profile.handle, db.handle, _dev_ptr(ids), n, _stream_ptr(stream), _dev_ptr(nats)),
+           "hmg_forward")
+
+
+def hmg_pipeline_forward(profile: Profile, db: Database, msv_raw, vit_raw, flags, survivor_ids, n_survivors,
+                         fwd_nats, fwd_ids, n_fwd, F1: float = 0.02, F2: float = 1e-3, stream=None):
+    """MSV -> compaction -> Viterbi -> compaction of the Viterbi passes -> Forward (Fig 1)."""
+    _check(lib().hmg_pipeline_forward(profile.handle, db.handle, F1, F2, _stream_ptr(stream), _dev_ptr(msv_raw),
+                                      _dev_ptr(vit_raw), _dev_ptr(flags), _dev_ptr(survivor_ids),
+                                      _dev_ptr(n_survivors), _dev_ptr(fwd_nats), _dev_ptr(fwd_ids),
+                                      _dev_ptr(n_fwd)), "hmg_pipeline_forward")
+
+
 def hmg_msv_nats(raw: int, L: int) -> float:
     return lib().hmg_msv_nats(int(raw), int(L))
 
@@ -265,7 +285,7 @@ def hmg_gumbel_surv(bits: float, mu: float, lam: float) -> float:
     return lib().hmg_gumbel_surv(bits, mu, lam)
 
 
-STAGES = ("msv_kernel", "msv_redo", "msv_flags_compaction", "vit_kernel", "vit_flags")
+STAGES = ("msv_kernel", "msv_redo", "msv_flags_compaction", "vit_kernel", "vit_flags", "fwd")
 
 
 def hmg_kernel_launches() -> int:
@@ -277,7 +297,7 @@ def hmg_set_stage_timing(enable: bool = True):
 
 
 def hmg_stage_times() -> dict:
-    ms = np.zeros(5, dtype=np.float64)
+    ms = np.zeros(len(STAGES), dtype=np.float64)
     _check(lib().hmg_stage_times(_np_ptr(ms)), "hmg_stage_times")
     return dict(zip(STAGES, ms.tolist()))
 
@@ -300,3 +320,12 @@ def alloc_outputs(nseq: int, device: int = 0):
                 flags=torch.zeros(nseq, dtype=torch.uint8, device=dev),
                 survivor_ids=torch.zeros(max(nseq, 1), dtype=torch.int32, device=dev),
                 n_survivors=torch.zeros(1, dtype=torch.int64, device=dev))
+
+
+def alloc_forward_outputs(nseq: int, device: int = 0):
+    """Extra caller-owned device outputs of hmg_pipeline_forward."""
+    import torch
+    dev = torch.device("cuda", device)
+    return dict(fwd_nats=torch.full((nseq,), float("nan"), dtype=torch.float32, device=dev),
+                fwd_ids=torch.zeros(max(nseq, 1), dtype=torch.int32, device=dev),
+                n_fwd=torch.zeros(1, dtype=torch.int64, device=dev))
