@@ -107,6 +107,8 @@ __global__ void __launch_bounds__(W * 32 > 256 ? W * 32 : 256, 1) fwd_kernel(con
     for (int q = 0; q < Q; ++q) Mc[q] = Ic[q] = Dc[q] = 0.0f;
     float xN = 1.0f, xJ = 0.0f, xC = 0.0f, xB = move;
     int scale_exp = 0;                          // accumulated log2 of the rescalings
+    bool row0 = true;                           // row 1: the diagonal carries are row 0's zeros
+    float csc = 1.0f;                           // rescale applied after cbuf was written (row i-1)
     const int nw = (L + 5) / 6;
     for (int w0 = 0; w0 < nw; w0 += 32) {
       const uint32_t wreg = (w0 + lane < nw) ? __ldg(wp + w0 + lane) : 0u;
@@ -140,8 +142,8 @@ __global__ void __launch_bounds__(W * 32 > 256 ? W * 32 : 256, 1) fwd_kernel(con
           float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
           float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
           if (lane == 0) {
-            if (W > 1 && w > 0) {
-              cM = cbuf[3 * (w - 1)]; cI = cbuf[3 * (w - 1) + 1]; cD = cbuf[3 * (w - 1) + 2];
+            if (W > 1 && w > 0 && !row0) {
+              cM = cbuf[3 * (w - 1)] * csc; cI = cbuf[3 * (w - 1) + 1] * csc; cD = cbuf[3 * (w - 1) + 2] * csc;
             } else {
               cM = cI = cD = 0.0f;
             }
@@ -209,15 +211,18 @@ __global__ void __launch_bounds__(W * 32 > 256 ? W * 32 : 256, 1) fwd_kernel(con
           xN *= loop;
           xJ = fmaf(xJ, loop, 0.5f * xE);
           xC = fmaf(xC, loop, 0.5f * xE);
+          csc = 1.0f;
           if (xE > kFwdRescale) {                // exact power-of-two rescale of the whole row
             const int ex = ilogbf(xE);
             const float sc = __int_as_float((127 - ex) << 23);
 #pragma unroll
             for (int q = 0; q < Q; ++q) { Mc[q] *= sc; Ic[q] *= sc; Dc[q] *= sc; }
             xN *= sc; xJ *= sc; xC *= sc;
+            csc = sc;                            // cbuf still holds the unscaled row
             scale_exp += ex;
           }
           xB = (xN + xJ) * move;
+          row0 = false;
         }
       }
     }
