@@ -78,6 +78,7 @@ typedef struct {
   int fwd_warps, fwd_nodes;         /* Forward kernel geometry: warps per sequence W, nodes per thread Q
                                        (0 = no Forward stage: no tsc, or M > 4096) */
   int fwd_rows_smem;                /* emission-odds rows staged in shared memory (the rest via L1) */
+  int fwd_seqs_per_block;           /* Forward kernel: sequences per block sharing the staged table */
 } hmg_quant;
 
 /* ---------------------------------------------------------------- profile */

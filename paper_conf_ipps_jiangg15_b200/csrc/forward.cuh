@@ -1,0 +1,211 @@
+// forward.cuh -- the Forward-stage kernel fwd_kernel<W, Q, S> (see forward.cu for the model,
+// the design and the host side).  W warps score one sequence, each thread owns Q contiguous
+// nodes, a block holds S sequences sharing one shared-memory copy of the emission odds.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "hmg_internal.h"
+
+namespace hmg {
+
+constexpr float kFwdRescale = 1099511627776.0f;   // 2^40: E above this triggers a rescale
+
+
+template <int Q> struct FwdVec { static constexpr int V = Q >= 4 ? 4 : Q; };
+
+__device__ __forceinline__ void group_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// Per-thread scan constants (host-computed from tDD, fwd_tables): the D->D carry into thread t is
+// c_in(t) = sum_{j<t} b_j prod_{j<m<t} a_m with a_m = prod of thread m's tDD and b_j its chain
+// from zero, so every slope in the scan is a profile constant and only the b's move per row.
+//   0..4  mul_d   slope of lanes (t-d, t] for the Hillis-Steele step d = 1, 2, 4, 8, 16
+//   5     pa      slope of lanes [warp start, t)        6  ai  slope of lanes [warp start, t]
+//   7     G       sum_{t'>t} Psum(t') prod_{t<m<t'} a_m  (E = sum_t [sum_q (M + Dloc) + b_t G_t])
+//   8     pa P_{Q-1}
+//   9..   P_q     prod_{q'<q} tDD_{q'} within the thread (D_q = Dloc_q + c_in P_q)
+constexpr int kFwdConst = 9;
+
+template <int W, int Q, int S>
+__global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
+  constexpr int T = 32 * W;                    // threads per sequence
+  constexpr int BT = T * S;                    // threads per block (S sequences)
+  constexpr int V = FwdVec<Q>::V;              // floats per vector load
+  constexpr int C = Q / V;                     // chunks per thread
+  constexpr int ROWF = T * Q;                  // floats per residue row
+  constexpr int PAR = (7 * W + 3) / 4 * 4;     // floats per parity buffer of a group (16-B aligned)
+  extern __shared__ float4 smem4[];
+  float* tab = reinterpret_cast<float*>(smem4);                   // [rows_smem][C][T][V]
+  const int g = threadIdx.x / T, t = threadIdx.x % T, w = t >> 5, lane = t & 31;
+  float* grp = tab + (size_t)a.rows_smem * ROWF + (size_t)g * (2 * PAR + 4);
+  int* slot = reinterpret_cast<int*>(grp + 2 * PAR);
+  const int bar = 1 + g;
+
+  {  // stage the emission odds (rows x < rows_smem) once per block
+    const float4* src = reinterpret_cast<const float4*>(a.etab);
+    float4* dst = reinterpret_cast<float4*>(tab);
+    const int n4 = a.rows_smem * ROWF / 4;
+    for (int i = threadIdx.x; i < n4; i += BT) dst[i] = src[i];
+  }
+  float tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q], P[Q];
+#pragma unroll
+  for (int q = 0; q < Q; ++q) {
+    const float* p = a.tr + (size_t)t * Q + q;
+    tBM[q] = p[0 * T * Q]; tMM[q] = p[1 * T * Q]; tIM[q] = p[2 * T * Q]; tDM[q] = p[3 * T * Q];
+    tMD[q] = p[4 * T * Q]; tMI[q] = p[5 * T * Q]; tII[q] = p[6 * T * Q]; tDD[q] = p[7 * T * Q];
+    P[q] = a.cst[(kFwdConst + q) * T + t];
+  }
+  float mul[5];
+#pragma unroll
+  for (int d = 0; d < 5; ++d) mul[d] = a.cst[d * T + t];
+  const float pa = a.cst[5 * T + t], ai = a.cst[6 * T + t], G = a.cst[7 * T + t], paP = a.cst[8 * T + t];
+  __syncthreads();
+
+  const int64_t n = a.list ? *a.nlist : a.nseq;
+  int par = 0;
+  for (;;) {
+    int64_t idx;
+    if constexpr (W == 1) {
+      unsigned long long v = 0;
+      if (lane == 0) v = atomicAdd(a.counter, 1ull);
+      idx = (int64_t)__shfl_sync(0xffffffffu, v, 0);
+    } else {
+      if (t == 0) *slot = (int)atomicAdd(a.counter, 1ull);
+      group_sync(bar, T);
+      idx = *slot;
+      group_sync(bar, T);
+    }
+    if (idx >= n) break;
+    const int s = a.list ? a.list[idx] : (int)idx;
+    const int L = a.len[s];
+    const uint32_t* wp = a.words + (size_t)a.woff16[s] * 4;
+    const float loop = (float)((double)L / (double)(L + 3));
+    const float move = (float)(3.0 / (double)(L + 3));
+    float Mc[Q], Ic[Q], Dc[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) Mc[q] = Ic[q] = Dc[q] = 0.0f;
+    float nM = 0.0f, nI = 0.0f, nD = 0.0f;     // lane 0 of warp w > 0: row i-1 cells of node t Q
+    float xN = 1.0f, xJ = 0.0f, xC = 0.0f, xB = move;
+    int scale_exp = 0;                          // accumulated log2 of the rescalings
+    const int nw = (L + 5) / 6;
+    for (int w0 = 0; w0 < nw; w0 += 32) {
+      const uint32_t wreg = (w0 + lane < nw) ? __ldg(wp + w0 + lane) : 0u;
+      const int wend = min(32, nw - w0);
+#pragma unroll 1
+      for (int j = 0; j < wend; ++j) {
+        const uint32_t word = __shfl_sync(0xffffffffu, wreg, j);
+        const int bend = min(6, L - 6 * (w0 + j));
+#pragma unroll 1
+        for (int b = 0; b < bend; ++b) {
+          const int x = (word >> (5 * b)) & 31;
+          float e[Q];
+          {
+            const float* er = (x < a.rows_smem ? tab : a.etab) + (size_t)x * ROWF;
+#pragma unroll
+            for (int c = 0; c < C; ++c) {
+              if constexpr (V == 4) {
+                const float4 v = reinterpret_cast<const float4*>(er)[c * T + t];
+                e[4 * c] = v.x; e[4 * c + 1] = v.y; e[4 * c + 2] = v.z; e[4 * c + 3] = v.w;
+              } else if constexpr (V == 2) {
+                const float2 v = reinterpret_cast<const float2*>(er)[c * T + t];
+                e[2 * c] = v.x; e[2 * c + 1] = v.y;
+              } else {
+                e[c] = er[c * T + t];
+              }
+            }
+          }
+          // diagonal carries: row i-1 cells of node t Q (thread t-1)
+          float cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
+          float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
+          float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
+          if (lane == 0) { cM = nM; cI = nI; cD = nD; }
+          // M and I from row i-1 (descending q: index q-1 still holds row i-1); B enters last
+#pragma unroll
+          for (int q = Q - 1; q >= 0; --q) {
+            const float pm = q ? Mc[q - 1] : cM;
+            const float pi = q ? Ic[q - 1] : cI;
+            const float pd = q ? Dc[q - 1] : cD;
+            float m = pm * tMM[q];
+            m = fmaf(pi, tIM[q], m);
+            m = fmaf(pd, tDM[q], m);
+            m = fmaf(xB, tBM[q], m);
+            Ic[q] = fmaf(Mc[q], tMI[q], Ic[q] * tII[q]);
+            Mc[q] = m * e[q];
+          }
+          // D->D within the thread from a zero carry (Dloc), the thread's contribution to E
+          float bsum = 0.0f, econ = 0.0f;
+#pragma unroll
+          for (int q = 0; q < Q; ++q) {
+            Dc[q] = bsum;
+            econ += Mc[q] + bsum;
+            bsum = fmaf(bsum, tDD[q], Mc[q] * tMD[q]);
+          }
+          econ = fmaf(bsum, G, econ);
+          // scan of the chain outputs (constant slopes) and the E reduction, independent chains
+          float ib = bsum;
+#pragma unroll
+          for (int d = 0; d < 5; ++d) {
+            const float ub = __shfl_up_sync(0xffffffffu, ib, 1 << d);
+            econ += __shfl_xor_sync(0xffffffffu, econ, 16 >> d);
+            if (lane >= (1 << d)) ib = fmaf(mul[d], ub, ib);
+          }
+          const float pb = __shfl_up_sync(0xffffffffu, ib, 1);
+          float xE = econ, cw = 0.0f;
+          if constexpr (W > 1) {
+            float* buf = grp + par * PAR;
+            float4* cbuf = reinterpret_cast<float4*>(buf);           // [W] last node M, I, D decomposition
+            float2* agg = reinterpret_cast<float2*>(buf + 4 * W);    // [W] (slope, b) of each warp
+            float* epart = buf + 6 * W;                              // [W]
+            if (lane == 31) {
+              agg[w] = make_float2(ai, ib);
+              cbuf[w] = make_float4(Mc[Q - 1], Ic[Q - 1], fmaf(pb, P[Q - 1], Dc[Q - 1]), paP);
+            }
+            if (lane == 0) epart[w] = econ;
+            group_sync(bar, T);
+            xE = 0.0f;
+#pragma unroll
+            for (int v = 0; v < W; ++v) xE += epart[v];
+            float cprev = 0.0f;
+            for (int v = 0; v < w; ++v) {
+              cprev = cw;
+              const float2 p = agg[v];
+              cw = fmaf(p.x, cw, p.y);
+            }
+            if (lane == 0 && w > 0) {
+              const float4 c = cbuf[w - 1];
+              nM = c.x; nI = c.y; nD = fmaf(c.w, cprev, c.z);
+            }
+            par ^= 1;
+          }
+          const float cin = lane == 0 ? cw : fmaf(pa, cw, pb);
+#pragma unroll
+          for (int q = 0; q < Q; ++q) Dc[q] = fmaf(cin, P[q], Dc[q]);
+          // specials (every thread, identical values)
+          xN *= loop;
+          xJ = fmaf(xJ, loop, 0.5f * xE);
+          xC = fmaf(xC, loop, 0.5f * xE);
+          if (xE > kFwdRescale) {                // exact power-of-two rescale of the whole row
+            const int ex = ilogbf(xE);
+            const float sc = __int_as_float((127 - ex) << 23);
+#pragma unroll
+            for (int q = 0; q < Q; ++q) { Mc[q] *= sc; Ic[q] *= sc; Dc[q] *= sc; }
+            nM *= sc; nI *= sc; nD *= sc;
+            xN *= sc; xJ *= sc; xC *= sc;
+            scale_exp += ex;
+          }
+          xB = (xN + xJ) * move;
+        }
+      }
+    }
+    if (t == 0) {
+      const double sc = (double)xC * (double)move;
+      const int c = a.order[s];
+      a.out[c] = sc > 0.0 ? (float)(log(sc) + (double)scale_exp * 0.6931471805599453) : -INFINITY;
+      if (a.flags) a.flags[c] |= 8u;
+    }
+  }
+}
+
+}  // namespace hmg

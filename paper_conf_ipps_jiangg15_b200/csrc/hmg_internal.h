@@ -90,6 +90,7 @@ struct FwdArgs {
   int64_t nseq;
   const float* etab;           // [kRows][C][T][V] emission odds (chunked), full copy in global memory
   const float* tr;             // [8][T][Q] transition odds
+  const float* cst;            // [kFwdConst + Q][T] D->D scan constants (forward.cu)
   int rows_smem;               // residue rows staged in shared memory (x < rows_smem)
   float* out;                  // [nseq] caller order, nats
   uint8_t* flags;              // [nseq] caller order or NULL: bit 3 set when the Forward stage ran
@@ -132,10 +133,11 @@ struct hmg_profile {
   int32_t* d_long_rsc = nullptr;
   int32_t* d_long_tr = nullptr;
   // Forward stage (forward.cu): fwd_kernel<fwd_W, fwd_Q>, emission rows x < fwd_rows in shared memory
-  int fwd_W = 0, fwd_Q = 0, fwd_rows = 0;
+  int fwd_W = 0, fwd_Q = 0, fwd_rows = 0, fwd_S = 1;   // S sequences per block
   float msc_max = 0.f;              // largest emission log-odds (odds-space range check)
   float* d_fwd_e = nullptr;         // emission odds [kRows][C][T][V]
   float* d_fwd_t = nullptr;         // transition odds [8][T][Q]
+  float* d_fwd_c = nullptr;         // D->D scan constants [kFwdConst + Q][T]
   // threshold caches (built on first use per F and DB Lmax)
   std::mutex mu;
   struct Thr {
@@ -203,10 +205,11 @@ cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* 
 
 // Forward stage (forward.cu)
 bool fwd_geometry(int M, int* W, int* Q);
-size_t fwd_smem(int W, int Q, int rows);
+size_t fwd_smem(int W, int Q, int rows, int S);
+int fwd_pick_s(int W, int Q, int rows);
 void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
-                std::vector<float>* tr);
-cudaError_t launch_fwd(int W, int Q, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok);
+                std::vector<float>* tr, std::vector<float>* cst);
+cudaError_t launch_fwd(int W, int Q, int S, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok);
 cudaError_t to_sorted_ids(const int32_t* caller_ids, int64_t n, const int32_t* inv_order, int32_t* sorted_ids,
                           cudaStream_t st);
 cudaError_t set_count(int64_t* d, int64_t v, cudaStream_t st);

@@ -784,8 +784,15 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     if (device >= 0) cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
     else smax = 227 * 1024;
     int rows = kAlpha;
-    while (rows > 0 && fwd_smem(p->fwd_W, p->fwd_Q, rows) > (size_t)smax) --rows;
+    while (rows > 0 && fwd_smem(p->fwd_W, p->fwd_Q, rows, 1) > (size_t)smax) --rows;
     p->fwd_rows = rows;
+    if (device >= 0) {
+      Dev dg(device);
+      p->fwd_S = fwd_pick_s(p->fwd_W, p->fwd_Q, rows);
+      const int so = env_int("HMG_FWD_S", 0);
+      if (so > 0) p->fwd_S = so;
+      if (p->fwd_S == 0) p->fwd_W = 0;   // no launchable configuration: Forward unsupported
+    }
   }
   // ---- kernel geometry and device tables
   p->msv_fast = p->bias < 66 + p->tbm;   // precondition of the fast MSV kernel
@@ -945,10 +952,11 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     }
   }
   if (st == HMG_OK && p->fwd_W > 0) {
-    std::vector<float> e, t;
-    fwd_tables(M, p->fwd_W, p->fwd_Q, msc, tsc, &e, &t);
+    std::vector<float> e, t, c;
+    fwd_tables(M, p->fwd_W, p->fwd_Q, msc, tsc, &e, &t, &c);
     st = upload(&p->d_fwd_e, e.data(), e.size());
     if (st == HMG_OK) st = upload(&p->d_fwd_t, t.data(), t.size());
+    if (st == HMG_OK) st = upload(&p->d_fwd_c, c.data(), c.size());
   }
   if (st != HMG_OK) {
     hmg_profile_destroy(p);
@@ -1046,6 +1054,7 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->fwd_warps = p->fwd_W;
   q->fwd_nodes = p->fwd_Q;
   q->fwd_rows_smem = p->fwd_rows;
+  q->fwd_seqs_per_block = p->fwd_S;
   return HMG_OK;
 }
 
@@ -1064,6 +1073,7 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_pair_tr);
     cudaFree(p->d_fwd_e);
     cudaFree(p->d_fwd_t);
+    cudaFree(p->d_fwd_c);
     cudaFree(p->thr_msv.d);
     cudaFree(p->thr_vit.d);
     cudaGetLastError();
@@ -1408,12 +1418,13 @@ static hmg_status run_fwd(const hmg_profile* p, const hmg_db* db, const int32_t*
   a.nseq = db->nseq;
   a.etab = p->d_fwd_e;
   a.tr = p->d_fwd_t;
+  a.cst = p->d_fwd_c;
   a.rows_smem = p->fwd_rows;
   a.out = nats;
   a.flags = flags;
   a.counter = ctr;
   int ok = 0;
-  if ((e = launch_fwd(p->fwd_W, p->fwd_Q, p->fwd_rows, a, st, &ok))) return cuda_status(e);
+  if ((e = launch_fwd(p->fwd_W, p->fwd_Q, p->fwd_S, p->fwd_rows, a, st, &ok))) return cuda_status(e);
   return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 

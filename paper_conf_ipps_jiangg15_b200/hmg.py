@@ -32,7 +32,8 @@ class hmg_quant(ctypes.Structure):
                 ("tsc", ctypes.POINTER(ctypes.c_int16)), ("msv_fast", c_int), ("msv_lanes", c_int),
                 ("msv_regs", c_int), ("vit_lanes", c_int), ("vit_nodes", c_int),
                 ("vit_pair_lanes", c_int), ("vit_pair_regs", c_int),
-                ("fwd_warps", c_int), ("fwd_nodes", c_int), ("fwd_rows_smem", c_int)]
+                ("fwd_warps", c_int), ("fwd_nodes", c_int), ("fwd_rows_smem", c_int),
+                ("fwd_seqs_per_block", c_int)]
 
 
 # name -> (restype, argtypes), exactly the declarations of include/hmg.h

@@ -225,3 +225,18 @@ def test_pipeline_forward_config3_full_size():
     dsq, off = db.materialize()
     nf = _check_pipeline_forward(prof, dsq, off, F1=0.02, F2=1e-3, sample=400)
     assert nf >= 400
+
+
+@pytest.mark.parametrize("M,S", [(40, 2), (40, 4), (40, 8), (40, 12), (200, 2), (200, 12), (300, 1), (300, 2),
+                                 (300, 4), (300, 6), (700, 1), (700, 2), (700, 3)])
+def test_fwd_every_block_shape(M, S, monkeypatch):
+    """Every instantiated (W, Q, S): S sequences per block share the staged table and take
+    sequences from the queue independently (named barriers per sequence group)."""
+    monkeypatch.setenv("HMG_FWD_S", str(S))
+    rng = np.random.default_rng(M * 100 + S)
+    prof = synth.make_profile(M, 9600 + M, dd=(1.0, 9.0))
+    dsq, off = _ragged(rng, n=90, lmax=400)
+    got, p = _fwd_gpu(prof.msc, prof.tsc, dsq, off)
+    assert p.quant()["fwd_seqs_per_block"] == S
+    want = oracle.fwd_db(prof.msc, prof.tsc, dsq, off)
+    _assert_close(got, want, np.diff(off), M)

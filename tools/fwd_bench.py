@@ -24,6 +24,6 @@ for M in Ms:
         hmg.hmg_forward(P, D, out)
         ts.append(hmg.hmg_stage_times()["fwd"])
     t = min(ts)
-    print(json.dumps({"M": M, "nseq": D.nseq, "residues": D.residues, "W": q["fwd_warps"], "Q": q["fwd_nodes"],
+    print(json.dumps({"M": M, "nseq": D.nseq, "residues": D.residues, "W": q["fwd_warps"], "Q": q["fwd_nodes"], "S": q["fwd_seqs_per_block"],
                       "rows_smem": q["fwd_rows_smem"], "ms": round(t, 3),
                       "gcups": round(M * D.residues / t / 1e6, 1)}), flush=True)
