@@ -36,6 +36,17 @@ sys.path.insert(0, ROOT)
 METRIC = "MSV / P7Viterbi / pipeline GCUPS at 1/2/4/8 B200; fraction of int-SIMD roofline"
 ALU_LANES_PER_CLK_SM = 64        # measured: VIADDMNMX/VIMNMX3 issue at 64 lanes/clk/SM (profiles/intpeak)
 MSV_ALU_OPS_PER_CELL = 0.75      # VIADDMNMX.S16x2 (1 per 2 cells) + VIMNMX3.S16x2 (1 per 4 cells)
+FP32_LANES_PER_CLK_SM = 128      # B200 FP32 FMA lanes per SM per clock (4 SMSPs x 32)
+FWD_FLOPS_PER_CELL = 16          # Forward recurrence: M 4 mul + 3 add + 1 mul, I 2 mul + 1 add,
+                                 # D 2 mul + 1 add, E 2 add
+
+
+def load_traffic(kernel):
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "traffic_r01.json")))[kernel]
+        return t["bytes"], t["source"]
+    except Exception:
+        return None, None
 
 
 def env_rank():
@@ -196,6 +207,7 @@ def main():
     ap.add_argument("--F2", type=float, default=1e-3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-forward", action="store_true")
     ap.add_argument("--cpu-sample-every", type=int, default=11)
     ap.add_argument("--ref-sample", type=int, default=20000)
     args = ap.parse_args()
@@ -299,11 +311,52 @@ def main():
     roofline = {"bound": "alu", "kernel": "msv_fast_kernel (+ concurrent long lane, one MSV stage)",
                 "achieved": round(achieved, 3), "peak": round(p_int, 3),
                 "unit": "T int-lane-ops/s", "frac": round(achieved / p_int, 4),
-                "traffic": None, "peak_source": "%s sm_max_mhz x %d SMs x %d lanes/clk (ALU pipe, measured "
+                "traffic": load_traffic("msv_fast_kernel")[0], "traffic_unit": "bytes/launch (ncu DRAM read+write)",
+                "traffic_source": load_traffic("msv_fast_kernel")[1], "peak_source": "%s sm_max_mhz x %d SMs x %d lanes/clk (ALU pipe, measured "
                                                 "profiles/intpeak)" % (src, nsm, ALU_LANES_PER_CLK_SM),
                 "algorithmic_ops_per_cell": MSV_ALU_OPS_PER_CELL, "kernel_cells": int(M * res_main),
                 "long_lane": {"sequences": nlong, "residues": res_long},
                 "kernel_ms": round(msv_ms, 4), "kernel_share_of_step": round(msv_ms / t_step, 4)}
+
+    # ---------------------------------------------------------------- Fig 1 with the Forward stage
+    # The same step followed by compaction of the Viterbi passes and the Forward kernel on them
+    # (hmg_pipeline_forward), timed the same way; reported beside the 8(a) headline, not in it.
+    forward = None
+    if not args.no_forward and world == 1 and P.quant()["fwd_warps"] > 0:
+        fo = hmg.alloc_forward_outputs(n, local)
+        hmg.hmg_set_stage_timing(True)
+        f_ms, f_stage = [], []
+        for i in range(args.warmup + args.steps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            hmg.hmg_pipeline_forward(P, D, F1=args.F1, F2=args.F2, stream=stream, **out, **fo)
+            b.record(stream)
+            sf = hmg.hmg_stage_times()["fwd"]
+            torch.cuda.synchronize()
+            if i >= args.warmup:
+                f_ms.append(a.elapsed_time(b))
+                f_stage.append(sf)
+        hmg.hmg_set_stage_timing(False)
+        nf = int(fo["n_fwd"].item())
+        fres = int(D.lengths[fo["fwd_ids"][:nf].cpu().numpy()].sum()) if nf else 0
+        tf, tfs = statistics.mean(f_ms), statistics.mean(f_stage)
+        q = P.quant()
+        fp_peak = FP32_LANES_PER_CLK_SM * 2 * nsm * f_peak / 1e12                # TFLOP/s (FMA = 2)
+        f_ach = FWD_FLOPS_PER_CELL * M * fres / (tfs * 1e-3) / 1e12 if tfs > 0 else 0.0
+        forward = {"sequences": nf, "residues": fres, "stage_ms": round(tfs, 4),
+                   "gcups": round(M * fres / (tfs * 1e-3) / 1e9, 2) if tfs > 0 else None,
+                   "fig1_pipeline_ms": round(tf, 4),
+                   "fig1_pipeline_gcups": round(M * res_local / (tf * 1e-3) / 1e9, 3),
+                   "kernel": "fwd_kernel<%d, %d, %d>" % (q["fwd_warps"], q["fwd_nodes"], q["fwd_seqs_per_block"]),
+                   "roofline": {"bound": "fp32", "achieved": round(f_ach, 3), "peak": round(fp_peak, 3),
+                                "unit": "TFLOP/s", "frac": round(f_ach / fp_peak, 4),
+                                "traffic": load_traffic("fwd_kernel")[0],
+                                "algorithmic_flops_per_cell": FWD_FLOPS_PER_CELL,
+                                "peak_source": "%s sm_max_mhz x %d SMs x %d FP32 lanes x 2 (FMA)"
+                                               % (src, nsm, FP32_LANES_PER_CLK_SM),
+                                "note": "stage = Viterbi-pass compaction + Forward kernel on %d sequences "
+                                        "(latency-bound at this size; tools/fwd_bench.py for throughput)" % nf}}
 
     # ---------------------------------------------------------------- end to end through the C ABI (host buffers)
     e2e = None
@@ -358,6 +411,7 @@ def main():
                        "survivors": int(ns_all), "survivor_frac": round(ns_all / max(n_all, 1), 5),
                        "survivor_residues": int(surv_all)},
             "roofline": roofline,
+            "forward": forward,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches),
