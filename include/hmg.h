@@ -208,6 +208,18 @@ hmg_status hmg_pipeline_forward(const hmg_profile* p, const hmg_db* db, double F
                                 uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
                                 int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids, int64_t* n_fwd);
 
+/* Many-profile MSV (the hmmscan / Pfam-scale workload): every
+ * (profile, sequence) pair of nprof profiles x the DB in one call, one kernel launch per bucket of
+ * profiles with a shared lane geometry (profiles padded to the bucket's largest model, <= 20%
+ * padding).  Work items are (DB chunk, profile) in chunk-major order, so the longest sequences of
+ * every profile start first and a chunk's residues stay in L2 while all profiles read them.
+ *   profs : host array [nprof] of profiles on the DB's device (1 <= nprof <= 65535; repeats allowed).
+ *   raw   : device uint8 [nprof][nseq], row i = profs[i], caller order: raw xJ as hmg_msv.
+ *   pass  : device uint8 [nprof][nseq] or NULL: 1 iff P_msv <= F1 (every profile needs ev).
+ * Results are identical to nprof hmg_msv calls (exact integer DP). */
+hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, void* stream,
+                         uint8_t* raw, uint8_t* pass);
+
 /* ---------------------------------------------------------------- instrumentation */
 
 /* Number of CUDA kernels this library has launched since it was loaded. */

@@ -39,6 +39,37 @@ struct MsvArgs {
   uint8_t* scratch;          // exact kernel: per-warp row buffers
 };
 
+// Many-profile MSV (msv_multi.cuh): a bucket of profiles with one lane geometry
+struct MsvMultiArgs {
+  MsvArgs base;              // DB fields (words, woff16, len, nseq, tjb); bias/tbm/raw set per profile
+  int nprof;
+  const uint32_t* const* prof;  // [nprof] striped tables in the bucket's (G, Q) layout
+  const int* bias;           // [nprof]
+  const int* tbm;            // [nprof]
+  uint8_t* raw;              // [nprof][nseq] sorted order (row p of the bucket)
+  long long nchunks;
+  int chunk;                 // sequences per chunk
+  unsigned long long* counter;
+};
+
+// exact MSV over (profile, sequence) pairs (msv_multi.cu): list entry j = p * nseq + s
+struct MsvPairArgs {
+  const uint32_t* words;
+  const uint32_t* woff16;
+  const int32_t* len;
+  int64_t nseq;
+  const uint8_t* tjb;
+  const uint8_t* const* cost;   // [nprof] plain biased costs [kRows][M_p]
+  const int* M;
+  const int* bias;
+  const int* tbm;
+  const int64_t* list;
+  const int64_t* nlist;
+  uint8_t* raw;              // [nprof][nseq] sorted order
+  uint8_t* scratch;          // per-warp rows, 2 (Mmax + 1) bytes each
+  int Mmax;
+};
+
 // ---------------------------------------------------------------- Viterbi kernel arguments
 struct VitArgs {
   const uint32_t* words;
@@ -138,6 +169,12 @@ struct hmg_profile {
   float* d_fwd_e = nullptr;         // emission odds [kRows][C][T][V]
   float* d_fwd_t = nullptr;         // transition odds [8][T][Q]
   float* d_fwd_c = nullptr;         // D->D scan constants [kFwdConst + Q][T]
+  // many-profile MSV (hmg_msv_batch): striped tables in other lane geometries, built on first use
+  struct Tab {
+    int G, Q;
+    uint32_t* d;
+  };
+  std::vector<Tab> msv_tabs;
   // threshold caches (built on first use per F and DB Lmax)
   std::mutex mu;
   struct Thr {
@@ -190,6 +227,15 @@ int long_msv_q(int M);
 int msv_q_max(int G);
 int msv_table_words(int G, int Q);   // MsvLayout<G, Q>::WORDS
 int vit_q_max(int G);
+
+// many-profile MSV (msv_multi.cu)
+cudaError_t launch_msv_multi(int G, int Q, const MsvMultiArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_msv_pairs_exact(const MsvPairArgs& a, int nwarps, cudaStream_t st);
+cudaError_t select_redo_pairs(const uint8_t* raw_sorted, int64_t n, int64_t* list, int64_t* count,
+                              cudaStream_t st);
+cudaError_t msv_flags_multi(const uint8_t* raw_sorted, int nprof, const int32_t* len, const int32_t* order,
+                            int64_t nseq, const uint16_t* const* thr, const int* rowmap, uint8_t* raw_out,
+                            uint8_t* pass_out, cudaStream_t st);
 
 // pipeline helpers (pipeline.cu)
 cudaError_t select_redo(const uint8_t* raw_sorted, int64_t n, int32_t* list, int64_t* count, void* tmp,

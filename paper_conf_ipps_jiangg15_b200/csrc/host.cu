@@ -1083,6 +1083,7 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_fwd_e);
     cudaFree(p->d_fwd_t);
     cudaFree(p->d_fwd_c);
+    for (auto& t : p->msv_tabs) cudaFree(t.d);
     cudaFree(p->thr_msv.d);
     cudaFree(p->thr_vit.d);
     cudaGetLastError();
@@ -1501,4 +1502,226 @@ hmg_status hmg_pipeline_forward(const hmg_profile* pc, const hmg_db* db, double 
   if (s != HMG_OK) return s;
   return cuda_status(cudaGetLastError());
 }
+
+// ------------------------------------------------------------------ many-profile MSV (f4)
+constexpr int kSideStreams = 8;
+
+// Per-device pool of non-blocking side streams (created on first use, kept for the process).
+static cudaStream_t* side_streams(int device) {
+  static std::mutex mu;
+  static std::vector<std::vector<cudaStream_t>> pools;
+  std::lock_guard<std::mutex> g(mu);
+  if ((int)pools.size() <= device) pools.resize(device + 1);
+  auto& v = pools[device];
+  if (v.empty()) {
+    for (int k = 0; k < kSideStreams; ++k) {
+      cudaStream_t s = nullptr;
+      if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) {
+        cudaGetLastError();
+        for (auto x : v) cudaStreamDestroy(x);
+        v.clear();
+        return nullptr;
+      }
+      v.push_back(s);
+    }
+  }
+  return v.data();
+}
+
+// Striped table of profile p in lane geometry (G, Q): its own table when the geometry matches,
+// else built on first use and cached in the profile (guarded by its mutex).
+static hmg_status msv_table_for(hmg_profile* p, int G, int Q, const uint32_t** out) {
+  if (G == p->msv_G && Q == p->msv_Q && p->d_msv_prof) {
+    *out = p->d_msv_prof;
+    return HMG_OK;
+  }
+  std::lock_guard<std::mutex> g(p->mu);
+  for (auto& t : p->msv_tabs)
+    if (t.G == G && t.Q == Q) {
+      *out = t.d;
+      return HMG_OK;
+    }
+  auto h = msv_table(*p, G, Q);
+  uint32_t* d = nullptr;
+  hmg_status s = upload(&d, h.data(), h.size());
+  if (s != HMG_OK) return s;
+  p->msv_tabs.push_back({G, Q, d});
+  *out = d;
+  return HMG_OK;
+}
+
+hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, void* stream,
+                         uint8_t* raw, uint8_t* pass) {
+  if (!profs || nprof < 1 || nprof > 65535 || !db || db->device < 0 || (!raw && db->nseq)) return HMG_EINVAL;
+  if (pass && !(F1 > 0.0 && F1 <= 1.0)) return HMG_EINVAL;
+  for (int i = 0; i < nprof; ++i) {
+    if (!profs[i] || profs[i]->device != db->device) return HMG_EINVAL;
+    if (pass && !profs[i]->has_ev) return HMG_EINVAL;
+  }
+  if (db->nseq == 0) return HMG_OK;
+  Dev dg(db->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t n = db->nseq;
+  // buckets: profiles sorted by M (descending); a bucket takes the geometry of its largest model
+  // and every following profile whose own register count at that G is >= (100 - pad)% of it
+  // (padding waste <= pad%); profiles outside the fast kernel's precondition go to the exact
+  // pair kernel
+  std::vector<int> idx;
+  std::vector<int> slow;
+  for (int i = 0; i < nprof; ++i) {
+    hmg_profile* p = const_cast<hmg_profile*>(profs[i]);
+    if (p->msv_fast && p->msv_Q > 0) idx.push_back(i);
+    else slow.push_back(i);
+  }
+  std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return profs[a]->M > profs[b]->M; });
+  struct Bucket { int G, Q, r0, r1; };
+  std::vector<Bucket> buckets;
+  std::vector<int> rows;                        // row r of the raw matrix -> caller profile index
+  // (measured, profiles/batch_bench_r01.jsonl: padding pays on small DBs -- fewer, fuller
+  //  launches -- and costs ~5% of cells on large ones, where every bucket fills the GPU anyway)
+  const bool large = n >= 50000;
+  const int pad_pct = env_int("HMG_MSV_BATCH_PAD", large ? 0 : 20);
+  for (size_t j = 0; j < idx.size();) {
+    int G = 0, Q = 0;
+    msv_geometry(profs[idx[j]]->M, &G, &Q);
+    const int r0 = (int)rows.size();
+    while (j < idx.size()) {
+      const int qj = (profs[idx[j]]->M + 2 * G) / (2 * G);
+      if ((int)rows.size() > r0 && 100 * qj < (100 - pad_pct) * Q) break;
+      rows.push_back(idx[j]);
+      ++j;
+    }
+    buckets.push_back({G, Q, r0, (int)rows.size()});
+  }
+  const int nfast = (int)rows.size();
+  for (int i : slow) rows.push_back(i);
+  // per-row arrays (bucket order)
+  std::vector<const uint32_t*> tabs(nprof, nullptr);
+  std::vector<const uint8_t*> costs(nprof);
+  std::vector<const uint16_t*> thr(nprof, nullptr);
+  std::vector<int> Ms(nprof), bias(nprof), tbm(nprof);
+  int Mmax = 0;
+  for (int r = 0; r < nprof; ++r) {
+    hmg_profile* p = const_cast<hmg_profile*>(profs[rows[r]]);
+    costs[r] = p->d_cost;
+    Ms[r] = p->M;
+    bias[r] = p->bias;
+    tbm[r] = p->tbm;
+    Mmax = std::max(Mmax, p->M);
+    if (pass) {
+      hmg_status s = msv_thr_table(p, db, F1, &thr[r]);
+      if (s != HMG_OK) return s;
+    }
+  }
+  for (const auto& b : buckets)
+    for (int r = b.r0; r < b.r1; ++r) {
+      hmg_status s = msv_table_for(const_cast<hmg_profile*>(profs[rows[r]]), b.G, b.Q, &tabs[r]);
+      if (s != HMG_OK) return s;
+    }
+  cudaError_t e = cudaSuccess;
+  {
+    Scratch S(st);
+    auto* raw_sorted = (uint8_t*)S.get((size_t)nprof * (size_t)n, &e);
+    auto* d_tabs = (const uint32_t**)S.get(sizeof(void*) * nprof, &e);
+    auto* d_costs = (const uint8_t**)S.get(sizeof(void*) * nprof, &e);
+    auto* d_thr = (const uint16_t**)S.get(sizeof(void*) * nprof, &e);
+    auto* d_ints = (int*)S.get(sizeof(int) * 4 * nprof, &e);
+    auto* list = (int64_t*)S.get(sizeof(int64_t) * (size_t)nprof * (size_t)n, &e);
+    auto* cnt = (int64_t*)S.get(sizeof(int64_t), &e);
+    const int nwarps_exact = 148 * 16;
+    auto* scr = (uint8_t*)S.get((size_t)nwarps_exact * 2 * (Mmax + 1), &e);
+    if (e) return cuda_status(e);
+    std::vector<int> ints;
+    ints.insert(ints.end(), Ms.begin(), Ms.end());
+    ints.insert(ints.end(), bias.begin(), bias.end());
+    ints.insert(ints.end(), tbm.begin(), tbm.end());
+    ints.insert(ints.end(), rows.begin(), rows.end());
+    if ((e = cudaMemcpyAsync(d_tabs, tabs.data(), sizeof(void*) * nprof, cudaMemcpyHostToDevice, st)) ||
+        (e = cudaMemcpyAsync(d_costs, costs.data(), sizeof(void*) * nprof, cudaMemcpyHostToDevice, st)) ||
+        (e = cudaMemcpyAsync(d_thr, thr.data(), sizeof(void*) * nprof, cudaMemcpyHostToDevice, st)) ||
+        (e = cudaMemcpyAsync(d_ints, ints.data(), sizeof(int) * 4 * nprof, cudaMemcpyHostToDevice, st)))
+      return cuda_status(e);
+    const int* d_M = d_ints;
+    const int* d_bias = d_ints + nprof;
+    const int* d_tbm = d_ints + 2 * nprof;
+    const int* d_rows = d_ints + 3 * nprof;
+    if (nfast < nprof &&   // profiles outside the fast precondition: every pair to the exact kernel
+        (e = cudaMemsetAsync(raw_sorted + (size_t)nfast * n, 254, (size_t)(nprof - nfast) * n, st)))
+      return cuda_status(e);
+    mark_reset();
+    mark(0, st);
+    auto* ctr = (unsigned long long*)S.get(sizeof(unsigned long long) * std::max<size_t>(buckets.size(), 1), &e);
+    if (e) return cuda_status(e);
+    if ((e = cudaMemsetAsync(ctr, 0, sizeof(unsigned long long) * std::max<size_t>(buckets.size(), 1), st)))
+      return cuda_status(e);
+    // buckets run concurrently on a pool of side streams (forked from and joined back into st), so
+    // one bucket's tail -- its longest sequences -- overlaps the other buckets' work
+    const int nside = (int)std::min<size_t>(buckets.size(), kSideStreams);
+    cudaStream_t* side = nside > 1 ? side_streams(db->device) : nullptr;
+    if (nside > 1 && !side) return HMG_ECUDA;
+    cudaEvent_t fork = nullptr, join[kSideStreams] = {};
+    if (nside > 1) {
+      if ((e = cudaEventCreateWithFlags(&fork, cudaEventDisableTiming))) return cuda_status(e);
+      if ((e = cudaEventRecord(fork, st))) return cuda_status(e);
+      for (int k = 0; k < nside; ++k) {
+        if ((e = cudaStreamWaitEvent(side[k], fork, 0))) return cuda_status(e);
+        if ((e = cudaEventCreateWithFlags(&join[k], cudaEventDisableTiming))) return cuda_status(e);
+      }
+    }
+    for (size_t bi = 0; bi < buckets.size(); ++bi) {
+      const Bucket& b = buckets[bi];
+      cudaStream_t bs = nside > 1 ? side[bi % nside] : st;
+      MsvMultiArgs m{};
+      m.base = msv_args(profs[rows[b.r0]], db);
+      m.nprof = b.r1 - b.r0;
+      m.prof = d_tabs + b.r0;
+      m.bias = d_bias + b.r0;
+      m.tbm = d_tbm + b.r0;
+      m.raw = raw_sorted + (size_t)b.r0 * n;
+      // chunk = R rounds of the block's 8 warps x 32/G sequences: large R keeps the item-boundary
+      // idling of a block's warps small (large DBs), R = 4 measured best on config-1-sized DBs
+      const int per_round = (32 / b.G) * 8;
+      const int R = env_int("HMG_MSV_BATCH_ROUNDS", large ? 16 : 4);
+      m.chunk = per_round * R;
+      m.nchunks = (n + m.chunk - 1) / m.chunk;
+      m.counter = ctr + bi;
+      int ok = 0;
+      if ((e = launch_msv_multi(b.G, b.Q, m, bs, &ok))) return cuda_status(e);
+      if (!ok) return HMG_EUNSUPPORTED;
+    }
+    if (nside > 1) {
+      for (int k = 0; k < nside; ++k) {
+        if ((e = cudaEventRecord(join[k], side[k]))) return cuda_status(e);
+        if ((e = cudaStreamWaitEvent(st, join[k], 0))) return cuda_status(e);
+        cudaEventDestroy(join[k]);
+      }
+      cudaEventDestroy(fork);
+    }
+    mark(1, st);
+    // exact re-score of the flagged pairs
+    if ((e = select_redo_pairs(raw_sorted, (int64_t)nprof * n, list, cnt, st))) return cuda_status(e);
+    MsvPairArgs x{};
+    x.words = db->d_words;
+    x.woff16 = db->d_woff16;
+    x.len = db->d_len;
+    x.nseq = n;
+    x.tjb = db->d_tjb;
+    x.cost = d_costs;
+    x.M = d_M;
+    x.bias = d_bias;
+    x.tbm = d_tbm;
+    x.list = list;
+    x.nlist = cnt;
+    x.raw = raw_sorted;
+    x.scratch = scr;
+    x.Mmax = Mmax;
+    if ((e = launch_msv_pairs_exact(x, nwarps_exact, st))) return cuda_status(e);
+    mark(2, st);
+    e = msv_flags_multi(raw_sorted, nprof, db->d_len, db->d_order, n, pass ? d_thr : nullptr, d_rows, raw, pass, st);
+    mark(3, st);
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  return cuda_status(e);
+}
+
 }  // extern "C"

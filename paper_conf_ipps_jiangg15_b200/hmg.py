@@ -55,6 +55,7 @@ SIGNATURES = {
     "hmg_pipeline": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_forward": (c_int, [c_p, c_p, c_p, c_i64, c_p, c_p]),
     "hmg_pipeline_forward": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
+    "hmg_msv_batch": (c_int, [c_p, c_int, c_p, c_d, c_p, c_p, c_p]),
     "hmg_msv_nats": (c_f, [c_int, c_int]),
     "hmg_vit_nats": (c_f, [c_int, c_int]),
     "hmg_null1_nats": (c_f, [c_int]),
@@ -268,6 +269,13 @@ def hmg_pipeline_forward(profile: Profile, db: Database, msv_raw, vit_raw, flags
                                       _dev_ptr(vit_raw), _dev_ptr(flags), _dev_ptr(survivor_ids),
                                       _dev_ptr(n_survivors), _dev_ptr(fwd_nats), _dev_ptr(fwd_ids),
                                       _dev_ptr(n_fwd)), "hmg_pipeline_forward")
+
+
+def hmg_msv_batch(profiles, db: Database, raw, pass_=None, F1: float = 0.02, stream=None):
+    """Many-profile MSV (f4): raw (uint8 [nprof][nseq]) and pass_ for every (profile, sequence) pair."""
+    arr = (c_p * len(profiles))(*[p.handle for p in profiles])
+    _check(lib().hmg_msv_batch(arr, len(profiles), db.handle, F1, _stream_ptr(stream), _dev_ptr(raw),
+                               _dev_ptr(pass_)), "hmg_msv_batch")
 
 
 def hmg_msv_nats(raw: int, L: int) -> float:
