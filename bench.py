@@ -208,6 +208,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-forward", action="store_true")
+    ap.add_argument("--batch", type=int, default=64, help="profiles of the f4 batch leg (0 = skip)")
     ap.add_argument("--cpu-sample-every", type=int, default=11)
     ap.add_argument("--ref-sample", type=int, default=20000)
     args = ap.parse_args()
@@ -358,6 +359,46 @@ def main():
                                 "note": "stage = Viterbi-pass compaction + Forward kernel on %d sequences "
                                         "(latency-bound at this size; tools/fwd_bench.py for throughput)" % nf}}
 
+    # ---------------------------------------------------------------- many-profile batch
+    # hmg_msv_batch of Pfam-like profiles (M ~ lognormal, median 180) over this rank's DB, one call per
+    # step, against one hmg_msv call per profile; reported beside the 8(a) headline, not in it.
+    batch = None
+    if args.batch > 0 and world == 1:
+        from paper_conf_ipps_jiangg15_b200 import synth as _synth
+        brng = np.random.default_rng(11)
+        bMs = np.clip(np.round(brng.lognormal(math.log(180), 0.6, size=args.batch)), 20, 1500).astype(int)
+        bprofs = [hmg.Profile(*(lambda q: (q.msc, q.tsc))(_synth.make_profile(int(m), 6000 + i)), device=local)
+                  for i, m in enumerate(bMs)]
+        braw = torch.empty((args.batch, n), dtype=torch.uint8, device=dev)
+
+        def btime(fn, k):
+            ts = []
+            for i in range(k + 1):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                fn()
+                b.record(stream)
+                torch.cuda.synchronize()
+                if i:
+                    ts.append(a.elapsed_time(b))
+            return statistics.mean(ts)
+
+        tb = btime(lambda: hmg.hmg_msv_batch(bprofs, D, braw, stream=stream), 3)
+
+        def loop():
+            for i, bp in enumerate(bprofs):
+                hmg.hmg_msv(bp, D, braw[i], stream=stream)
+
+        tl = btime(loop, 2)
+        bcells = int(bMs.sum()) * res_local
+        batch = {"profiles": args.batch, "sum_M": int(bMs.sum()), "cells": bcells, "ms": round(tb, 3),
+                 "gcups": round(bcells / (tb * 1e-3) / 1e9, 2), "per_profile_calls_ms": round(tl, 3),
+                 "per_profile_calls_gcups": round(bcells / (tl * 1e-3) / 1e9, 2),
+                 "speedup_vs_calls": round(tl / tb, 3),
+                 "workload": "hmg_msv_batch: %d Pfam-like profiles (M ~ lognormal median 180, 20..1500, seeds "
+                             "6000+i) x this DB; L2 flushed before each timed call" % args.batch}
+
     # ---------------------------------------------------------------- end to end through the C ABI (host buffers)
     e2e = None
     if not args.no_e2e and world == 1:
@@ -412,6 +453,7 @@ def main():
                        "survivor_residues": int(surv_all)},
             "roofline": roofline,
             "forward": forward,
+            "batch": batch,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches),
