@@ -208,6 +208,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-forward", action="store_true")
+    ap.add_argument("--no-graph", action="store_true", help="launch the pipeline eagerly in the timed region")
     ap.add_argument("--batch", type=int, default=64, help="profiles of the f4 batch leg (0 = skip)")
     ap.add_argument("--cpu-sample-every", type=int, default=11)
     ap.add_argument("--ref-sample", type=int, default=20000)
@@ -249,21 +250,43 @@ def main():
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
-    def step():
-        hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=stream, **out)
+    def pipeline(st):
+        hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=st, **out)
+
+    def gather():
         if world > 1:
             packed = hdist.pack_results(out["msv_raw"], out["vit_raw"], out["flags"])
             hdist.gather(packed, out["survivor_ids"], out["n_survivors"], gids, world)
+
+    for _ in range(args.warmup):                       # eager warm-up (threshold tables, module load)
+        pipeline(stream)
+        gather()
+    torch.cuda.synchronize()
+
+    # The pipeline is captured once in a CUDA graph (its 15 launches, scratch allocation and memsets
+    # become one graph launch: no host launch gaps between the stages); the NCCL gather stays eager.
+    graph, launches_per_step = None, None
+    if not args.no_graph:
+        graph = torch.cuda.CUDAGraph()
+        n0 = hmg.hmg_kernel_launches()
+        with torch.cuda.graph(graph):
+            pipeline(torch.cuda.current_stream())
+        launches_per_step = hmg.hmg_kernel_launches() - n0
+
+    def step():
+        if graph is not None:
+            graph.replay()
+        else:
+            pipeline(stream)
+        gather()
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
 
     # ---------------------------------------------------------------- timed region (device-resident inputs)
-    hmg.hmg_set_stage_timing(True)
     launches0 = hmg.hmg_kernel_launches()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    stages = []
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -273,13 +296,24 @@ def main():
             evs[i][0].record(stream)
             step()
             evs[i][1].record(stream)
-            stages.append(hmg.hmg_stage_times())       # waits for this step's last stage event
-            redo = hmg.hmg_stage_counts()["vit_pair_redo"]
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     launches = hmg.hmg_kernel_launches() - launches0
+    if graph is not None:
+        launches += launches_per_step * args.steps     # graph replays launch the captured kernels
+    # stage times: the same pipeline eagerly, with the library's stage events (not in the timed region)
+    hmg.hmg_set_stage_timing(True)
+    stages = []
+    for i in range(args.steps):
+        flush.zero_()
+        pipeline(stream)
+        stages.append(hmg.hmg_stage_times())           # waits for this call's last stage event
+        redo = hmg.hmg_stage_counts()["vit_pair_redo"]
     hmg.hmg_set_stage_timing(False)
+    if graph is not None:
+        graph.replay()                                 # leave the outputs of a timed-path step
+    torch.cuda.synchronize()
     ms = [a.elapsed_time(b) for a, b in evs]
     t_step = sum(ms) / len(ms)
     t_max = torch.tensor([t_step], dtype=torch.float64, device=dev)
@@ -409,16 +443,30 @@ def main():
         h_flags = torch.empty(n, dtype=torch.uint8, pin_memory=True)
         h_ns = torch.empty(1, dtype=torch.int64, pin_memory=True)
         e_ms = []
-        for i in range(args.warmup + args.steps):
-            flush.zero_()
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            D.upload(img, stream=stream)                                   # H2D of the packed DB
-            hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=stream, **out)
+
+        def e2e_step(st):
+            D.upload(img, stream=st)                                       # H2D of the packed DB
+            hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=st, **out)
             h_msv.copy_(out["msv_raw"], non_blocking=True)                 # D2H of the results
             h_vit.copy_(out["vit_raw"], non_blocking=True)
             h_flags.copy_(out["flags"], non_blocking=True)
             h_ns.copy_(out["n_survivors"], non_blocking=True)
+
+        e2e_graph = None
+        if graph is not None:                                              # same launch mode as the timed step
+            e2e_step(stream)
+            torch.cuda.synchronize()
+            e2e_graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(e2e_graph):
+                e2e_step(torch.cuda.current_stream())
+        for i in range(args.warmup + args.steps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            if e2e_graph is not None:
+                e2e_graph.replay()
+            else:
+                e2e_step(stream)
             b.record(stream)
             b.synchronize()
             if i >= args.warmup:
@@ -442,6 +490,8 @@ def main():
                        "M": M, "nseq_per_rank": n, "residues_per_rank": res_local, "nseq_total": int(n_all),
                        "residues_total": int(res_all), "F1": args.F1, "F2": args.F2,
                        "l2": "flushed (256 MiB write) before every timed step, outside its events",
+                       "launch": "CUDA graph of hmg_pipeline (captured once), replayed per step" if graph is not None
+                                 else "eager hmg_pipeline calls",
                        "parallelism": "db-shard x%d (snake length-balanced), NCCL all_gather of results" % world},
             "stages": {"msv_kernel_ms": round(msv_ms, 4), "msv_gcups": round(msv_gcups, 2),
                        "msv_redo_ms": round(st["msv_redo"], 4),
