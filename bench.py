@@ -269,7 +269,7 @@ def main():
     if not args.no_graph:
         graph = torch.cuda.CUDAGraph()
         n0 = hmg.hmg_kernel_launches()
-        with torch.cuda.graph(graph):
+        with torch.cuda.graph(graph, capture_error_mode="thread_local"):
             pipeline(torch.cuda.current_stream())
         launches_per_step = hmg.hmg_kernel_launches() - n0
 
@@ -457,7 +457,7 @@ def main():
             e2e_step(stream)
             torch.cuda.synchronize()
             e2e_graph = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(e2e_graph):
+            with torch.cuda.graph(e2e_graph, capture_error_mode="thread_local"):
                 e2e_step(torch.cuda.current_stream())
         for i in range(args.warmup + args.steps):
             flush.zero_()

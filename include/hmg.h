@@ -220,6 +220,17 @@ hmg_status hmg_pipeline_forward(const hmg_profile* p, const hmg_db* db, double F
 hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, void* stream,
                          uint8_t* raw, uint8_t* pass);
 
+/* The Fig 1 filter pipeline for every profile of a batch: hmg_msv_batch's MSV stage, then per
+ * profile (concurrently on side streams) pass flags + stable survivor compaction + the Viterbi
+ * filter on its survivors.  Outputs are hmg_pipeline's, one row per profile (row i = profs[i]):
+ *   msv_raw uint8 [nprof][nseq], vit_raw int16 [nprof][nseq] (survivors only), flags uint8
+ *   [nprof][nseq], survivor_ids int32 [nprof][nseq] (row i holds n_survivors[i] caller indices,
+ *   length-descending), n_survivors int64 [nprof] (device).
+ * Every profile needs tsc and ev.  Results equal nprof hmg_pipeline calls. */
+hmg_status hmg_pipeline_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, double F2,
+                              void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
+                              int32_t* survivor_ids, int64_t* n_survivors);
+
 /* ---------------------------------------------------------------- instrumentation */
 
 /* Number of CUDA kernels this library has launched since it was loaded. */

@@ -1550,15 +1550,29 @@ static hmg_status msv_table_for(hmg_profile* p, int G, int Q, const uint32_t** o
   return HMG_OK;
 }
 
-hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, void* stream,
-                         uint8_t* raw, uint8_t* pass) {
+// Outputs of the batched pipeline tail (hmg_pipeline_batch): per-profile rows of [nprof][nseq].
+struct BatchTail {
+  double F2;
+  int16_t* vit_raw;
+  uint8_t* flags;
+  int32_t* survivor_ids;
+  int64_t* n_survivors;
+};
+
+static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1,
+                                 void* stream, uint8_t* raw, uint8_t* pass, const BatchTail* tail) {
   if (!profs || nprof < 1 || nprof > 65535 || !db || db->device < 0 || (!raw && db->nseq)) return HMG_EINVAL;
-  if (pass && !(F1 > 0.0 && F1 <= 1.0)) return HMG_EINVAL;
+  if ((pass || tail) && !(F1 > 0.0 && F1 <= 1.0)) return HMG_EINVAL;
   for (int i = 0; i < nprof; ++i) {
     if (!profs[i] || profs[i]->device != db->device) return HMG_EINVAL;
-    if (pass && !profs[i]->has_ev) return HMG_EINVAL;
+    if ((pass || tail) && !profs[i]->has_ev) return HMG_EINVAL;
+    if (tail && !profs[i]->has_tsc) return HMG_EINVAL;
   }
-  if (db->nseq == 0) return HMG_OK;
+  if (db->nseq == 0) {
+    if (tail && tail->n_survivors)
+      return cuda_status(cudaMemsetAsync(tail->n_survivors, 0, sizeof(int64_t) * nprof, (cudaStream_t)stream));
+    return HMG_OK;
+  }
   Dev dg(db->device);
   cudaStream_t st = (cudaStream_t)stream;
   const int64_t n = db->nseq;
@@ -1608,7 +1622,7 @@ hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_d
     bias[r] = p->bias;
     tbm[r] = p->tbm;
     Mmax = std::max(Mmax, p->M);
-    if (pass) {
+    if (pass || tail) {
       hmg_status s = msv_thr_table(p, db, F1, &thr[r]);
       if (s != HMG_OK) return s;
     }
@@ -1717,11 +1731,90 @@ hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_d
     x.Mmax = Mmax;
     if ((e = launch_msv_pairs_exact(x, nwarps_exact, st))) return cuda_status(e);
     mark(2, st);
-    e = msv_flags_multi(raw_sorted, nprof, db->d_len, db->d_order, n, pass ? d_thr : nullptr, d_rows, raw, pass, st);
-    mark(3, st);
+    if (!tail) {
+      e = msv_flags_multi(raw_sorted, nprof, db->d_len, db->d_order, n, pass ? d_thr : nullptr, d_rows, raw, pass,
+                          st);
+      mark(3, st);
+    } else {
+      // per profile (Fig 1): pass flags + stable survivor compaction of its row, Viterbi filter on the
+      // survivors, flags; the profiles' chains run concurrently on the side streams
+      std::vector<const int32_t*> tv(nprof);
+      for (int r = 0; r < nprof; ++r) {
+        hmg_status s = vit_thr_table(const_cast<hmg_profile*>(profs[rows[r]]), db, tail->F2, &tv[r]);
+        if (s != HMG_OK) return s;
+      }
+      const int ns = std::min(nprof, kSideStreams);
+      cudaStream_t* side = ns > 1 ? side_streams(db->device) : nullptr;
+      if (ns > 1 && !side) return HMG_ECUDA;
+      cudaEvent_t fork = nullptr, join[kSideStreams] = {};
+      if (ns > 1) {
+        if ((e = cudaEventCreateWithFlags(&fork, cudaEventDisableTiming))) return cuda_status(e);
+        if ((e = cudaEventRecord(fork, st))) return cuda_status(e);
+        for (int k = 0; k < ns; ++k) {
+          if ((e = cudaStreamWaitEvent(side[k], fork, 0))) return cuda_status(e);
+          if ((e = cudaEventCreateWithFlags(&join[k], cudaEventDisableTiming))) return cuda_status(e);
+        }
+      }
+      {
+        std::vector<Scratch*> SS;
+        struct Bufs { int32_t* surv; int16_t* vraw; void* tmp; };
+        std::vector<Bufs> B;
+        hmg_status s = HMG_OK;
+        for (int k = 0; k < std::max(ns, 1); ++k) {
+          cudaStream_t sk = ns > 1 ? side[k] : st;
+          SS.push_back(new Scratch(sk));
+          Bufs b{};
+          b.surv = (int32_t*)SS.back()->get(sizeof(int32_t) * (size_t)n, &e);
+          b.vraw = (int16_t*)SS.back()->get(sizeof(int16_t) * (size_t)n, &e);
+          b.tmp = SS.back()->get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
+          B.push_back(b);
+        }
+        for (int r = 0; r < nprof && !e && s == HMG_OK; ++r) {
+          const int k = ns > 1 ? r % ns : 0;
+          cudaStream_t sk = ns > 1 ? side[k] : st;
+          const int i = rows[r];
+          const hmg_profile* pi = profs[i];
+          const size_t ro = (size_t)i * n;
+          e = msv_finish(raw_sorted + (size_t)r * n, db->d_len, db->d_order, n, thr[r], raw + ro, tail->flags + ro,
+                         B[k].surv, tail->n_survivors + i, tail->survivor_ids + ro, B[k].tmp, sk);
+          if (e) break;
+          s = run_vit(pi, db, B[k].surv, tail->n_survivors + i, sk, B[k].vraw, *SS[k], nullptr, 0, false, n);
+          if (s != HMG_OK) break;
+          e = vit_finish(B[k].vraw, B[k].surv, tail->n_survivors + i, n, db->d_len, db->d_order, tv[r],
+                         tail->vit_raw + ro, nullptr, tail->flags + ro, sk);
+        }
+        for (auto* x : SS) delete x;                 // stream-ordered frees on each side stream
+        if (s != HMG_OK) return s;
+        if (e) return cuda_status(e);
+      }
+      if (ns > 1) {
+        for (int k = 0; k < ns; ++k) {
+          if ((e = cudaEventRecord(join[k], side[k]))) return cuda_status(e);
+          if ((e = cudaStreamWaitEvent(st, join[k], 0))) return cuda_status(e);
+          cudaEventDestroy(join[k]);
+        }
+        cudaEventDestroy(fork);
+      }
+      mark(5, st);
+    }
   }
   if (e == cudaSuccess) e = cudaGetLastError();
   return cuda_status(e);
+}
+
+hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, void* stream,
+                         uint8_t* raw, uint8_t* pass) {
+  return msv_batch_impl(profs, nprof, db, F1, stream, raw, pass, nullptr);
+}
+
+hmg_status hmg_pipeline_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, double F2,
+                              void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
+                              int32_t* survivor_ids, int64_t* n_survivors) {
+  if (!(F2 > 0.0 && F2 <= 1.0)) return HMG_EINVAL;
+  if (db && db->nseq && (!vit_raw || !flags || !survivor_ids || !n_survivors)) return HMG_EINVAL;
+  if (db && !db->nseq && !n_survivors) return HMG_EINVAL;
+  BatchTail t{F2, vit_raw, flags, survivor_ids, n_survivors};
+  return msv_batch_impl(profs, nprof, db, F1, stream, msv_raw, nullptr, &t);
 }
 
 }  // extern "C"

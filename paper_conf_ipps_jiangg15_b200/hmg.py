@@ -56,6 +56,7 @@ SIGNATURES = {
     "hmg_forward": (c_int, [c_p, c_p, c_p, c_i64, c_p, c_p]),
     "hmg_pipeline_forward": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_batch": (c_int, [c_p, c_int, c_p, c_d, c_p, c_p, c_p]),
+    "hmg_pipeline_batch": (c_int, [c_p, c_int, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_nats": (c_f, [c_int, c_int]),
     "hmg_vit_nats": (c_f, [c_int, c_int]),
     "hmg_null1_nats": (c_f, [c_int]),
@@ -276,6 +277,26 @@ def hmg_msv_batch(profiles, db: Database, raw, pass_=None, F1: float = 0.02, str
     arr = (c_p * len(profiles))(*[p.handle for p in profiles])
     _check(lib().hmg_msv_batch(arr, len(profiles), db.handle, F1, _stream_ptr(stream), _dev_ptr(raw),
                                _dev_ptr(pass_)), "hmg_msv_batch")
+
+
+def hmg_pipeline_batch(profiles, db: Database, msv_raw, vit_raw, flags, survivor_ids, n_survivors,
+                       F1: float = 0.02, F2: float = 1e-3, stream=None):
+    """Fig 1 filter pipeline for every profile of a batch (f4); outputs are [nprof][nseq] rows."""
+    arr = (c_p * len(profiles))(*[p.handle for p in profiles])
+    _check(lib().hmg_pipeline_batch(arr, len(profiles), db.handle, F1, F2, _stream_ptr(stream), _dev_ptr(msv_raw),
+                                    _dev_ptr(vit_raw), _dev_ptr(flags), _dev_ptr(survivor_ids),
+                                    _dev_ptr(n_survivors)), "hmg_pipeline_batch")
+
+
+def alloc_batch_outputs(nprof: int, nseq: int, device: int = 0):
+    """Caller-owned device outputs for hmg_pipeline_batch."""
+    import torch
+    dev = torch.device("cuda", device)
+    return dict(msv_raw=torch.zeros((nprof, nseq), dtype=torch.uint8, device=dev),
+                vit_raw=torch.full((nprof, nseq), -32768, dtype=torch.int16, device=dev),
+                flags=torch.zeros((nprof, nseq), dtype=torch.uint8, device=dev),
+                survivor_ids=torch.zeros((nprof, max(nseq, 1)), dtype=torch.int32, device=dev),
+                n_survivors=torch.zeros(nprof, dtype=torch.int64, device=dev))
 
 
 def hmg_msv_nats(raw: int, L: int) -> float:

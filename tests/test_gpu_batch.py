@@ -143,3 +143,33 @@ def test_batch_invalid_and_empty():
     assert ei.value.status == hmg.HMG_EINVAL
     with pytest.raises(hmg.HmgError):
         hmg.hmg_msv_batch([], db2, out)
+
+
+def test_pipeline_batch_equals_per_profile_pipelines():
+    """hmg_pipeline_batch (MSV batch -> per-profile compaction + Viterbi on side streams) equals one
+    hmg_pipeline call per profile on every output, and the oracle on the survivors of two rows."""
+    prof1, dbs = synth.config(1)
+    dsq, off = dbs.materialize()
+    lam = math.log(2)
+    Ms = (64, 150, 200, 420, 700, 1100, 64)
+    profs = [synth.make_profile(M, 6400 + i) for i, M in enumerate(Ms)]
+    evs = [(_mu_msv(pr), lam, _mu_msv(pr) - 1.0, lam) for pr in profs]
+    P = [hmg.Profile(pr.msc, pr.tsc, ev=ev) for pr, ev in zip(profs, evs)]
+    db = hmg.Database(dsq, off)
+    out = hmg.alloc_batch_outputs(len(P), db.nseq)
+    hmg.hmg_pipeline_batch(P, db, F1=0.1, F2=0.05, **out)
+    torch.cuda.synchronize()
+    for i, p in enumerate(P):
+        one = hmg.alloc_outputs(db.nseq)
+        hmg.hmg_pipeline(p, db, F1=0.1, F2=0.05, **one)
+        torch.cuda.synchronize()
+        ns = int(one["n_survivors"].item())
+        assert int(out["n_survivors"][i].item()) == ns > 0
+        assert torch.equal(out["msv_raw"][i], one["msv_raw"])
+        assert torch.equal(out["flags"][i], one["flags"])
+        assert torch.equal(out["survivor_ids"][i][:ns], one["survivor_ids"][:ns])
+        assert torch.equal(out["vit_raw"][i], one["vit_raw"])
+        if i in (0, 4):
+            sv = one["survivor_ids"][:ns].cpu().numpy()
+            want = oracle.vit_db(oracle.VitProfile(profs[i].msc, profs[i].tsc), dsq, off, ids=sv)
+            assert np.array_equal(out["vit_raw"][i].cpu().numpy().astype(np.int32)[sv], want)

@@ -45,3 +45,25 @@ for name, cfg in (("config1-db", 1), ("config2-db", 2)):
                       "sum_M": int(Ms.sum()), "cells": cells, "batch_ms": round(t_b, 3),
                       "batch_gcups": round(cells / t_b / 1e6, 1), "loop_ms": round(t_l, 3),
                       "loop_gcups": round(cells / t_l / 1e6, 1), "speedup": round(t_l / t_b, 2)}), flush=True)
+
+# Fig 1 pipeline for every profile (hmg_pipeline_batch) vs one hmg_pipeline call per profile
+evs = [p.calibrate() for p in profs]
+pprofs = [hmg.Profile(*(lambda q: (q.msc, q.tsc))(synth.make_profile(int(M), 6000 + i)), ev=evs[i])
+          for i, M in enumerate(Ms)]
+for name, cfg in (("config1-db", 1), ("config2-db", 2)):
+    _, dbs = synth.config(cfg)
+    dsq, off = dbs.materialize()
+    D = hmg.Database(dsq, off)
+    out = hmg.alloc_batch_outputs(P, D.nseq)
+    ones = [hmg.alloc_outputs(D.nseq) for _ in range(min(P, 8))]
+    cells = int(Ms.sum()) * D.residues
+    t_b = timed(lambda: hmg.hmg_pipeline_batch(pprofs, D, **out))
+    def loop():
+        for i, p in enumerate(pprofs):
+            hmg.hmg_pipeline(p, D, **ones[i % len(ones)])
+    t_l = timed(loop)
+    ns = out["n_survivors"].cpu().numpy()
+    print(json.dumps({"pipeline": True, "db": name, "nseq": D.nseq, "profiles": P, "cells": cells,
+                      "survivors_mean": float(ns.mean()), "batch_ms": round(t_b, 3),
+                      "batch_gcups": round(cells / t_b / 1e6, 1), "loop_ms": round(t_l, 3),
+                      "loop_gcups": round(cells / t_l / 1e6, 1), "speedup": round(t_l / t_b, 2)}), flush=True)
