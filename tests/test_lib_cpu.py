@@ -143,3 +143,35 @@ def test_conversions_match_oracle(L):
     for x in (-30.0, -5.0, 0.0, 3.3, 40.0):
         a, b = hmg.hmg_gumbel_surv(x, -9.0, math.log(2)), oracle.gumbel_surv(x, -9.0, math.log(2))
         assert a == b or abs(a - b) <= 1e-6 * abs(b)
+
+
+def test_host_only_handles_rejected_by_compute_calls(L):
+    """Compute entry points (incl. Forward and the batch calls) reject host-only handles and bad
+    arguments with HMG_EINVAL before touching a device (no GPU needed)."""
+    msc = np.zeros((8, 29), np.float32)
+    tsc = np.full((8, 8), -1.0, np.float32)
+    p = hmg.Profile(msc, tsc, device=-1)
+    d = hmg.Database(np.zeros(12, np.uint8), np.array([0, 5, 12]), device=-1)
+    q = p.quant()
+    assert q["fwd_warps"] == 1 and q["fwd_nodes"] == 2 and q["fwd_rows_smem"] == 29
+    vp = ctypes.c_void_p
+    assert L.hmg_forward(p.handle, d.handle, None, 0, None, vp(1)) == hmg.HMG_EINVAL
+    assert L.hmg_pipeline_forward(p.handle, d.handle, 0.02, 1e-3, None, vp(1), vp(1), vp(1), vp(1), vp(1),
+                                  vp(1), vp(1), vp(1)) == hmg.HMG_EINVAL
+    arr = (vp * 1)(p.handle)
+    assert L.hmg_msv_batch(arr, 1, d.handle, 0.02, None, vp(1), None) == hmg.HMG_EINVAL
+    assert L.hmg_msv_batch(arr, 0, d.handle, 0.02, None, vp(1), None) == hmg.HMG_EINVAL
+    assert L.hmg_pipeline_batch(arr, 1, d.handle, 0.02, 2.0, None, vp(1), vp(1), vp(1), vp(1),
+                                vp(1)) == hmg.HMG_EINVAL
+
+
+def test_forward_geometry_host_only(L):
+    """Forward kernel geometry: fewest warps at 8 nodes per thread, then fewest
+    nodes; unsupported above 4096 nodes."""
+    for M, (W, Qn) in {1: (1, 2), 64: (1, 2), 65: (1, 4), 129: (1, 8), 256: (1, 8), 257: (2, 8),
+                       400: (2, 8), 513: (4, 8), 1000: (4, 8), 2048: (8, 8), 4096: (16, 8)}.items():
+        p = hmg.Profile(np.zeros((M, 29), np.float32), np.full((M, 8), -1.0, np.float32), device=-1)
+        q = p.quant()
+        assert (q["fwd_warps"], q["fwd_nodes"]) == (W, Qn), M
+    p = hmg.Profile(np.zeros((4097, 29), np.float32), np.full((4097, 8), -1.0, np.float32), device=-1)
+    assert p.quant()["fwd_warps"] == 0
