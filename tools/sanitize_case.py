@@ -32,3 +32,28 @@ raw = torch.zeros(D.nseq, dtype=torch.uint8, device="cuda")
 hmg.hmg_msv(P, D, raw)
 torch.cuda.synchronize()
 print("exact ok")
+# Forward stage (every group width W with its block shape S) and the Fig 1 pipeline with Forward
+for M in (60, 300, 700, 1500):
+    prof = synth.make_profile(M, 50 + M, dd=(1.0, 9.0))
+    P = hmg.Profile(prof.msc, prof.tsc, ev=(-9.0, 0.693, -9.0, 0.693))
+    D = hmg.Database(dsq, off)
+    f = torch.zeros(D.nseq, dtype=torch.float32, device="cuda")
+    hmg.hmg_forward(P, D, f)
+    out = hmg.alloc_outputs(D.nseq)
+    fo = hmg.alloc_forward_outputs(D.nseq)
+    hmg.hmg_pipeline_forward(P, D, F1=0.5, F2=0.5, **out, **fo)
+    torch.cuda.synchronize()
+    print("forward M", M, "ok", int(fo["n_fwd"].item()))
+# many-profile batch (two buckets, a profile outside the fast precondition) and its pipeline
+profs = [synth.make_profile(M, 70 + M) for M in (40, 64, 300, 310)]
+Ps = [hmg.Profile(p.msc, p.tsc, ev=(-9.0, 0.693, -9.0, 0.693)) for p in profs]
+Ps.append(hmg.Profile(np.full((40, 29), 30.0, np.float32), np.full((40, 8), -1.0, np.float32),
+                      ev=(-9.0, 0.693, -9.0, 0.693)))
+D = hmg.Database(dsq, off)
+raw = torch.zeros((len(Ps), D.nseq), dtype=torch.uint8, device="cuda")
+pas = torch.zeros((len(Ps), D.nseq), dtype=torch.uint8, device="cuda")
+hmg.hmg_msv_batch(Ps, D, raw, pas, F1=0.5)
+ob = hmg.alloc_batch_outputs(len(Ps), D.nseq)
+hmg.hmg_pipeline_batch(Ps, D, F1=0.5, F2=0.5, **ob)
+torch.cuda.synchronize()
+print("batch ok", ob["n_survivors"].tolist())
