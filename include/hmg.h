@@ -76,7 +76,8 @@ typedef struct {
                                         the s32 kernel: lanes per sequence G, s16x2 registers Q per
                                         cell type; 0 = not used for this profile */
   int fwd_warps, fwd_nodes;         /* Forward kernel geometry: warps per sequence W, nodes per thread Q
-                                       (0 = no Forward stage: no tsc, or M > 4096) */
+                                       (Q = 16 up to 8 warps, else 8; 0 = no Forward stage: no tsc,
+                                       or M > 4096) */
   int fwd_rows_smem;                /* emission-odds rows staged in shared memory (the rest via L1) */
   int fwd_seqs_per_block;           /* Forward kernel: sequences per block sharing the staged table */
 } hmg_quant;

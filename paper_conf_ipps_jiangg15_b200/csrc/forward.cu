@@ -90,12 +90,14 @@ int fwd_pick_s(int W, int Q, int rows) {
   return best;
 }
 
-// Geometry: the fewest warps per sequence with 8 nodes per thread, then the fewest nodes per
-// thread (2, 4, 8) for that width; models above 4096 nodes are not supported by this kernel.
-bool fwd_geometry(int M, int* W, int* Q) {
+// Geometry: the fewest warps per sequence at qmax nodes per thread (16 for the lean variant, up
+// to 8 warps; else 8, up to 16 warps), then the fewest nodes per thread (2, 4, 8, 16) for that
+// width; models above 4096 nodes are not supported by this kernel.
+bool fwd_geometry(int M, int* W, int* Q, int qmax) {
+  const int wmax = qmax >= 16 ? 8 : 16;   // 16 nodes/thread: <= 256 threads per sequence (registers)
   int w = 1;
-  while (32 * w * 8 < M && w < 16) w *= 2;
-  if (32 * w * 8 < M) return false;
+  while (32 * w * qmax < M && w < wmax) w *= 2;
+  if (32 * w * qmax < M) return false;
   int q = 2;
   while (32 * w * q < M) q *= 2;
   *W = w;

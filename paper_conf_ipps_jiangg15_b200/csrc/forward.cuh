@@ -49,14 +49,20 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
     const int n4 = a.rows_smem * ROWF / 4;
     for (int i = threadIdx.x; i < n4; i += BT) dst[i] = src[i];
   }
-  float tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q], P[Q];
+  // LEAN (Q = 16): no per-node P registers; D = Dloc + c_in P is applied as two 8-node product
+  // chains (c_in and c_in P_8), keeping the thread at ~220 registers so one warp holds 512 nodes
+  constexpr bool LEAN = Q >= 16;
+  constexpr int NP = LEAN ? 1 : Q;
+  float tBM[Q], tMM[Q], tIM[Q], tDM[Q], tMD[Q], tMI[Q], tII[Q], tDD[Q], P[NP];
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     const float* p = a.tr + (size_t)t * Q + q;
     tBM[q] = p[0 * T * Q]; tMM[q] = p[1 * T * Q]; tIM[q] = p[2 * T * Q]; tDM[q] = p[3 * T * Q];
     tMD[q] = p[4 * T * Q]; tMI[q] = p[5 * T * Q]; tII[q] = p[6 * T * Q]; tDD[q] = p[7 * T * Q];
-    P[q] = a.cst[(kFwdConst + q) * T + t];
+    if constexpr (!LEAN) P[q] = a.cst[(kFwdConst + q) * T + t];
   }
+  if constexpr (LEAN) P[0] = a.cst[(kFwdConst + Q / 2) * T + t];   // P_{Q/2}
+  const float PL = a.cst[(kFwdConst + Q - 1) * T + t];             // P_{Q-1} (cross-warp carry)
   float mul[5];
 #pragma unroll
   for (int d = 0; d < 5; ++d) mul[d] = a.cst[d * T + t];
@@ -83,19 +89,12 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
     const uint32_t* wp = a.words + (size_t)a.woff16[s] * 4;
     const float loop = (float)((double)L / (double)(L + 3));
     const float move = (float)(3.0 / (double)(L + 3));
-    // Software-pipelined rows: iteration i finishes row i (D->D, E, specials) while the parts of row
-    // i+1 that need neither row i's D nor B_i -- the emission load, the M'tMM + I'tIM partials and
-    // the I update -- fill the latency of row i's shuffle scans and barrier; row i+1's M cells are
-    // completed at the end of the iteration.
-    float Mc[Q], Ic[Q], Dc[Q], mp[Q], e[Q];
+    float Mc[Q], Ic[Q], Dc[Q], e[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) Mc[q] = Ic[q] = Dc[q] = 0.0f;
+    float nM = 0.0f, nI = 0.0f, nD = 0.0f;     // lane 0 of warp w > 0: row i-1 cells of node t Q
     float xN = 1.0f, xJ = 0.0f, xC = 0.0f, xB = move;
     int scale_exp = 0;                          // accumulated log2 of the rescalings
-    // residue stream: words fetched 32 at a time (one per lane), one chunk ahead
-    const int nw = (L + 5) / 6;
-    uint32_t wcur = (lane < nw) ? __ldg(wp + lane) : 0u;
-    uint32_t wnxt = (32 + lane < nw) ? __ldg(wp + 32 + lane) : 0u;
-    int rj = 0, rb = 0, rw0 = 0;                // word in chunk, residue in word, chunk base
-    uint32_t word = __shfl_sync(0xffffffffu, wcur, 0);
     auto load_row = [&](const float* er, bool shared) {
 #pragma unroll
       for (int c = 0; c < C; ++c) {
@@ -110,115 +109,113 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
         }
       }
     };
-    // x is uniform over the group (>= one warp): shared-memory rows by LDS, the rest through L1
-    auto load_e = [&](int x) {
-      if (x < a.rows_smem) load_row(tab + (size_t)x * ROWF, true);
-      else load_row(a.etab + (size_t)x * ROWF, false);
-    };
-    // row 1 (row 0 is all zero): M = B_0 tBM e, I = D = 0
-    load_e(word & 31);
-#pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      Mc[q] = xB * tBM[q] * e[q];
-      Ic[q] = 0.0f;
-    }
+    const int nw = (L + 5) / 6;
+    for (int w0 = 0; w0 < nw; w0 += 32) {
+      const uint32_t wreg = (w0 + lane < nw) ? __ldg(wp + w0 + lane) : 0u;
+      const int wend = min(32, nw - w0);
 #pragma unroll 1
-    for (int i = 0; i < L; ++i) {
-      // next residue (row i+1; a dummy code 0 after the last row keeps the body branch-free)
-      if (++rb == 6) {
-        rb = 0;
-        if (++rj == 32) {
-          rj = 0;
-          rw0 += 32;
-          wcur = wnxt;
-          wnxt = (rw0 + 32 + lane < nw) ? __ldg(wp + rw0 + 32 + lane) : 0u;
+      for (int j = 0; j < wend; ++j) {
+        const uint32_t word = __shfl_sync(0xffffffffu, wreg, j);
+        const int bend = min(6, L - 6 * (w0 + j));
+#pragma unroll 1
+        for (int b = 0; b < bend; ++b) {
+          const int x = (word >> (5 * b)) & 31;
+          // x is uniform over the group (>= one warp): shared-memory rows by LDS, the rest via L1
+          if (x < a.rows_smem) load_row(tab + (size_t)x * ROWF, true);
+          else load_row(a.etab + (size_t)x * ROWF, false);
+          // diagonal carries: row i-1 cells of node t Q (thread t-1)
+          float cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
+          float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
+          float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
+          if (lane == 0) { cM = nM; cI = nI; cD = nD; }
+          // M and I from row i-1 (descending q: index q-1 still holds row i-1)
+#pragma unroll
+          for (int q = Q - 1; q >= 0; --q) {
+            const float pm = q ? Mc[q - 1] : cM;
+            const float pi = q ? Ic[q - 1] : cI;
+            const float pd = q ? Dc[q - 1] : cD;
+            float m = pm * tMM[q];
+            m = fmaf(pi, tIM[q], m);
+            m = fmaf(pd, tDM[q], m);
+            m = fmaf(xB, tBM[q], m);
+            Ic[q] = fmaf(Mc[q], tMI[q], Ic[q] * tII[q]);
+            Mc[q] = m * e[q];
+          }
+          // D->D within the thread from a zero carry (Dloc), the thread's contribution to E
+          float bsum = 0.0f, econ = 0.0f;
+#pragma unroll
+          for (int q = 0; q < Q; ++q) {
+            Dc[q] = bsum;
+            econ += Mc[q] + bsum;
+            bsum = fmaf(bsum, tDD[q], Mc[q] * tMD[q]);
+          }
+          econ = fmaf(bsum, G, econ);
+          // scan of the chain outputs (constant slopes) and the E reduction, independent chains
+          float ib = bsum;
+#pragma unroll
+          for (int d = 0; d < 5; ++d) {
+            const float ub = __shfl_up_sync(0xffffffffu, ib, 1 << d);
+            econ += __shfl_xor_sync(0xffffffffu, econ, 16 >> d);
+            if (lane >= (1 << d)) ib = fmaf(mul[d], ub, ib);
+          }
+          const float pb = __shfl_up_sync(0xffffffffu, ib, 1);
+          float xE = econ, cw = 0.0f;
+          if constexpr (W > 1) {
+            float* buf = grp + par * PAR;
+            float4* cbuf = reinterpret_cast<float4*>(buf);           // [W] last node M, I, D decomposition
+            float2* agg = reinterpret_cast<float2*>(buf + 4 * W);    // [W] (slope, b) of each warp
+            float* epart = buf + 6 * W;                              // [W]
+            if (lane == 31) {
+              agg[w] = make_float2(ai, ib);
+              cbuf[w] = make_float4(Mc[Q - 1], Ic[Q - 1], fmaf(pb, PL, Dc[Q - 1]), paP);
+            }
+            if (lane == 0) epart[w] = econ;
+            group_sync(bar, T);
+            xE = 0.0f;
+#pragma unroll
+            for (int v = 0; v < W; ++v) xE += epart[v];
+            float cprev = 0.0f;
+            for (int v = 0; v < w; ++v) {
+              cprev = cw;
+              const float2 pv = agg[v];
+              cw = fmaf(pv.x, cw, pv.y);
+            }
+            if (lane == 0 && w > 0) {
+              const float4 c = cbuf[w - 1];
+              nM = c.x; nI = c.y; nD = fmaf(c.w, cprev, c.z);
+            }
+            par ^= 1;
+          }
+          // row i's D: Dloc + c_in P
+          const float cin = lane == 0 ? cw : fmaf(pa, cw, pb);
+          if constexpr (LEAN) {
+            float c0 = cin, c1 = cin * P[0];
+#pragma unroll
+            for (int q = 0; q < Q / 2; ++q) {
+              Dc[q] += c0;
+              Dc[q + Q / 2] += c1;
+              c0 *= tDD[q];
+              c1 *= tDD[q + Q / 2];
+            }
+          } else {
+#pragma unroll
+            for (int q = 0; q < Q; ++q) Dc[q] = fmaf(cin, P[q], Dc[q]);
+          }
+          // specials (every thread, identical values)
+          xN *= loop;
+          xJ = fmaf(xJ, loop, 0.5f * xE);
+          xC = fmaf(xC, loop, 0.5f * xE);
+          if (xE > kFwdRescale) {                // exact power-of-two rescale of the whole row
+            const int ex = ilogbf(xE);
+            const float sc = __int_as_float((127 - ex) << 23);
+#pragma unroll
+            for (int q = 0; q < Q; ++q) { Mc[q] *= sc; Ic[q] *= sc; Dc[q] *= sc; }
+            nM *= sc; nI *= sc; nD *= sc;
+            xN *= sc; xJ *= sc; xC *= sc;
+            scale_exp += ex;
+          }
+          xB = (xN + xJ) * move;
         }
-        word = __shfl_sync(0xffffffffu, wcur, rj);
-      }
-      const int xn = i + 1 < L ? (int)((word >> (5 * rb)) & 31) : 0;
-      load_e(xn);
-      // D->D of row i within the thread from a zero carry (Dloc), its E contribution
-      float bsum = 0.0f, econ = 0.0f;
-#pragma unroll
-      for (int q = 0; q < Q; ++q) {
-        Dc[q] = bsum;
-        econ += Mc[q] + bsum;
-        bsum = fmaf(bsum, tDD[q], Mc[q] * tMD[q]);
-      }
-      econ = fmaf(bsum, G, econ);
-      // row i+1 partials from row i's M and I (node t Q's row-i cells from thread t-1)
-      const float McL = Mc[Q - 1], IcL = Ic[Q - 1];
-      float cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
-      float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
-#pragma unroll
-      for (int q = Q - 1; q >= 1; --q) {
-        mp[q] = fmaf(Ic[q - 1], tIM[q], Mc[q - 1] * tMM[q]);
-        Ic[q] = fmaf(Mc[q], tMI[q], Ic[q] * tII[q]);
-      }
-      Ic[0] = fmaf(Mc[0], tMI[0], Ic[0] * tII[0]);
-      // scan of the chain outputs (constant slopes) and the E reduction, independent chains
-      float ib = bsum;
-#pragma unroll
-      for (int d = 0; d < 5; ++d) {
-        const float ub = __shfl_up_sync(0xffffffffu, ib, 1 << d);
-        econ += __shfl_xor_sync(0xffffffffu, econ, 16 >> d);
-        if (lane >= (1 << d)) ib = fmaf(mul[d], ub, ib);
-      }
-      const float pb = __shfl_up_sync(0xffffffffu, ib, 1);
-      float xE = econ, cw = 0.0f, cDl = 0.0f;
-      if (lane == 0) cM = cI = 0.0f;
-      if constexpr (W > 1) {
-        float* buf = grp + par * PAR;
-        float4* cbuf = reinterpret_cast<float4*>(buf);           // [W] last node M, I, D decomposition
-        float2* agg = reinterpret_cast<float2*>(buf + 4 * W);    // [W] (slope, b) of each warp
-        float* epart = buf + 6 * W;                              // [W]
-        if (lane == 31) {
-          agg[w] = make_float2(ai, ib);
-          cbuf[w] = make_float4(McL, IcL, fmaf(pb, P[Q - 1], Dc[Q - 1]), paP);
-        }
-        if (lane == 0) epart[w] = econ;
-        group_sync(bar, T);
-        xE = 0.0f;
-#pragma unroll
-        for (int v = 0; v < W; ++v) xE += epart[v];
-        float cprev = 0.0f;
-        for (int v = 0; v < w; ++v) {
-          cprev = cw;
-          const float2 pv = agg[v];
-          cw = fmaf(pv.x, cw, pv.y);
-        }
-        if (lane == 0 && w > 0) {
-          const float4 c = cbuf[w - 1];
-          cM = c.x; cI = c.y; cDl = fmaf(c.w, cprev, c.z);
-        }
-        par ^= 1;
-      }
-      mp[0] = fmaf(cI, tIM[0], cM * tMM[0]);
-      // row i's D: Dloc + c_in P
-      const float cin = lane == 0 ? cw : fmaf(pa, cw, pb);
-#pragma unroll
-      for (int q = 0; q < Q; ++q) Dc[q] = fmaf(cin, P[q], Dc[q]);
-      // specials (every thread, identical values)
-      xN *= loop;
-      xJ = fmaf(xJ, loop, 0.5f * xE);
-      xC = fmaf(xC, loop, 0.5f * xE);
-      if (xE > kFwdRescale) {                  // exact power-of-two rescale of everything row i feeds
-        const int ex = ilogbf(xE);
-        const float sc = __int_as_float((127 - ex) << 23);
-#pragma unroll
-        for (int q = 0; q < Q; ++q) { mp[q] *= sc; Ic[q] *= sc; Dc[q] *= sc; }
-        cDl *= sc;
-        xN *= sc; xJ *= sc; xC *= sc;
-        scale_exp += ex;
-      }
-      xB = (xN + xJ) * move;
-      // complete row i+1's M cells: + D'_{k-1} tDM + B tBM, times the emission odds
-      float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
-      if (lane == 0) cD = cDl;
-#pragma unroll
-      for (int q = Q - 1; q >= 0; --q) {
-        const float pd = q ? Dc[q - 1] : cD;
-        Mc[q] = fmaf(xB, tBM[q], fmaf(pd, tDM[q], mp[q])) * e[q];
       }
     }
     if (t == 0) {

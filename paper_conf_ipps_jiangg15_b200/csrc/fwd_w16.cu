@@ -1,10 +1,11 @@
-// Instantiations of fwd_kernel<16, Q, S> for Q = 2, 4, 8 and S = 1.
+// Instantiations of fwd_kernel<16, Q, S> for Q = 2, 4, 8, 16 and S = 1.
 #include "forward.cuh"
 
 namespace hmg {
 namespace {
 template <int Q>
 const void* pick_s(int s) {
+  if (Q == 16 && 32 * 16 * s > 256) return nullptr;   // 16 nodes/thread need ~250 registers
   if (s == 1) return reinterpret_cast<const void*>(&fwd_kernel<16, Q, 1>);
   return nullptr;
 }
@@ -14,6 +15,7 @@ const void* fwd_ptr_w16(int q, int s) {
     case 2: return pick_s<2>(s);
     case 4: return pick_s<4>(s);
     case 8: return pick_s<8>(s);
+    case 16: return pick_s<16>(s);
   }
   return nullptr;
 }

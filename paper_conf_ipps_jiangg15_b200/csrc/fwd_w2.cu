@@ -1,10 +1,11 @@
-// Instantiations of fwd_kernel<2, Q, S> for Q = 2, 4, 8 and S = 1, 2, 4, 6.
+// Instantiations of fwd_kernel<2, Q, S> for Q = 2, 4, 8, 16 and S = 1, 2, 4, 6.
 #include "forward.cuh"
 
 namespace hmg {
 namespace {
 template <int Q>
 const void* pick_s(int s) {
+  if (Q == 16 && 32 * 2 * s > 256) return nullptr;   // 16 nodes/thread need ~250 registers
   if (s == 1) return reinterpret_cast<const void*>(&fwd_kernel<2, Q, 1>);
   if (s == 2) return reinterpret_cast<const void*>(&fwd_kernel<2, Q, 2>);
   if (s == 4) return reinterpret_cast<const void*>(&fwd_kernel<2, Q, 4>);
@@ -17,6 +18,7 @@ const void* fwd_ptr_w2(int q, int s) {
     case 2: return pick_s<2>(s);
     case 4: return pick_s<4>(s);
     case 8: return pick_s<8>(s);
+    case 16: return pick_s<16>(s);
   }
   return nullptr;
 }

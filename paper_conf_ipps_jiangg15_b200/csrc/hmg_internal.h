@@ -250,7 +250,7 @@ cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* 
                           int32_t* ids_caller, int64_t* count, void* tmp, cudaStream_t st);
 
 // Forward stage (forward.cu)
-bool fwd_geometry(int M, int* W, int* Q);
+bool fwd_geometry(int M, int* W, int* Q, int qmax);
 size_t fwd_smem(int W, int Q, int rows, int S);
 int fwd_pick_s(int W, int Q, int rows);
 void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::vector<float>* etab,

@@ -779,11 +779,12 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   p->msc_max = -INFINITY;
   for (size_t i = 0; i < (size_t)M * kAlpha; ++i) p->msc_max = std::max(p->msc_max, msc[i]);
   // ---- Forward stage geometry (forward.cu): emission rows staged in shared memory as fit
-  if (tsc && fwd_geometry(M, &p->fwd_W, &p->fwd_Q)) {
+  const int fwd_qmax = env_int("HMG_FWD_QMAX", 16) >= 16 ? 16 : 8;   // 16: profiles/fwd_bench_r01e.jsonl
+  if (tsc && (fwd_geometry(M, &p->fwd_W, &p->fwd_Q, fwd_qmax) || fwd_geometry(M, &p->fwd_W, &p->fwd_Q, 8))) {
     const int wo = env_int("HMG_FWD_W", 0);   // wider groups (shorter rows, more threads per sequence)
     if (wo == 1 || wo == 2 || wo == 4 || wo == 8 || wo == 16) {
       int q = 2;
-      while (32 * wo * q < M && q < 8) q *= 2;
+      while (32 * wo * q < M && q < 16) q *= 2;
       if (32 * wo * q >= M) {
         p->fwd_W = wo;
         p->fwd_Q = q;

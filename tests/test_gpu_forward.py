@@ -227,16 +227,34 @@ def test_pipeline_forward_config3_full_size():
     assert nf >= 400
 
 
-@pytest.mark.parametrize("M,S", [(40, 2), (40, 4), (40, 8), (40, 12), (200, 2), (200, 12), (300, 1), (300, 2),
-                                 (300, 4), (300, 6), (700, 1), (700, 2), (700, 3)])
-def test_fwd_every_block_shape(M, S, monkeypatch):
+@pytest.mark.parametrize("M,S,qmax", [(40, 2, 16), (40, 4, 16), (40, 8, 16), (40, 12, 16), (200, 2, 16),
+                                      (200, 12, 16), (300, 1, 8), (300, 2, 8), (300, 4, 8), (300, 6, 8),
+                                      (700, 1, 8), (700, 2, 8), (700, 3, 8), (300, 2, 16), (300, 4, 16),
+                                      (300, 8, 16), (700, 1, 16), (700, 2, 16), (700, 4, 16)])
+def test_fwd_every_block_shape(M, S, qmax, monkeypatch):
     """Every instantiated (W, Q, S): S sequences per block share the staged table and take
     sequences from the queue independently (named barriers per sequence group)."""
     monkeypatch.setenv("HMG_FWD_S", str(S))
+    monkeypatch.setenv("HMG_FWD_QMAX", str(qmax))
     rng = np.random.default_rng(M * 100 + S)
     prof = synth.make_profile(M, 9600 + M, dd=(1.0, 9.0))
     dsq, off = _ragged(rng, n=90, lmax=400)
     got, p = _fwd_gpu(prof.msc, prof.tsc, dsq, off)
     assert p.quant()["fwd_seqs_per_block"] == S
+    want = oracle.fwd_db(prof.msc, prof.tsc, dsq, off)
+    _assert_close(got, want, np.diff(off), M)
+
+
+@pytest.mark.parametrize("M", [100, 257, 400, 512, 513, 1000, 2048, 3000])
+def test_fwd_lean_sixteen_nodes(M, monkeypatch):
+    """The register-lean 16-nodes-per-thread variant (HMG_FWD_QMAX=16: one warp up to M = 512, no
+    per-row barrier; D = Dloc + c_in P applied as two 8-node product chains)."""
+    monkeypatch.setenv("HMG_FWD_QMAX", "16")
+    rng = np.random.default_rng(M + 77)
+    prof = synth.make_profile(M, 9700 + M, dd=(1.0, 9.0))
+    dsq, off = _ragged(rng, n=50, lmax=400)
+    got, p = _fwd_gpu(prof.msc, prof.tsc, dsq, off)
+    q = p.quant()
+    assert q["fwd_nodes"] == 16 or M <= 256
     want = oracle.fwd_db(prof.msc, prof.tsc, dsq, off)
     _assert_close(got, want, np.diff(off), M)

@@ -166,10 +166,10 @@ def test_host_only_handles_rejected_by_compute_calls(L):
 
 
 def test_forward_geometry_host_only(L):
-    """Forward kernel geometry: fewest warps at 8 nodes per thread, then fewest
+    """Forward kernel geometry: fewest warps at 16 nodes per thread, then fewest
     nodes; unsupported above 4096 nodes."""
-    for M, (W, Qn) in {1: (1, 2), 64: (1, 2), 65: (1, 4), 129: (1, 8), 256: (1, 8), 257: (2, 8),
-                       400: (2, 8), 513: (4, 8), 1000: (4, 8), 2048: (8, 8), 4096: (16, 8)}.items():
+    for M, (W, Qn) in {1: (1, 2), 64: (1, 2), 65: (1, 4), 129: (1, 8), 256: (1, 8), 257: (1, 16),
+                       400: (1, 16), 513: (2, 16), 1000: (2, 16), 2048: (4, 16), 4096: (8, 16)}.items():
         p = hmg.Profile(np.zeros((M, 29), np.float32), np.full((M, 8), -1.0, np.float32), device=-1)
         q = p.quant()
         assert (q["fwd_warps"], q["fwd_nodes"]) == (W, Qn), M
