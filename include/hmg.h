@@ -227,10 +227,13 @@ hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_d
  *   msv_raw uint8 [nprof][nseq], vit_raw int16 [nprof][nseq] (survivors only), flags uint8
  *   [nprof][nseq], survivor_ids int32 [nprof][nseq] (row i holds n_survivors[i] caller indices,
  *   length-descending), n_survivors int64 [nprof] (device).
- * Every profile needs tsc and ev.  Results equal nprof hmg_pipeline calls. */
+ * Optional Forward stage (all three NULL = off): fwd_nats float32 [nprof][nseq], fwd_ids int32
+ * [nprof][nseq], n_fwd int64 [nprof] as hmg_pipeline_forward per row (flags bit3).
+ * Every profile needs tsc and ev.  Results equal nprof hmg_pipeline (_forward) calls. */
 hmg_status hmg_pipeline_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, double F2,
                               void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
-                              int32_t* survivor_ids, int64_t* n_survivors);
+                              int32_t* survivor_ids, int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids,
+                              int64_t* n_fwd);
 
 /* ---------------------------------------------------------------- instrumentation */
 

@@ -1558,6 +1558,9 @@ struct BatchTail {
   uint8_t* flags;
   int32_t* survivor_ids;
   int64_t* n_survivors;
+  float* fwd_nats;           // optional Forward stage (all three or none)
+  int32_t* fwd_ids;
+  int64_t* n_fwd;
 };
 
 static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1,
@@ -1568,10 +1571,15 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
     if (!profs[i] || profs[i]->device != db->device) return HMG_EINVAL;
     if ((pass || tail) && !profs[i]->has_ev) return HMG_EINVAL;
     if (tail && !profs[i]->has_tsc) return HMG_EINVAL;
+    if (tail && tail->fwd_nats && (profs[i]->fwd_W == 0 || profs[i]->msc_max > kFwdMscMax)) return HMG_EUNSUPPORTED;
   }
   if (db->nseq == 0) {
-    if (tail && tail->n_survivors)
-      return cuda_status(cudaMemsetAsync(tail->n_survivors, 0, sizeof(int64_t) * nprof, (cudaStream_t)stream));
+    if (tail && tail->n_survivors) {
+      cudaError_t e0 = cudaMemsetAsync(tail->n_survivors, 0, sizeof(int64_t) * nprof, (cudaStream_t)stream);
+      if (e0 == cudaSuccess && tail->n_fwd)
+        e0 = cudaMemsetAsync(tail->n_fwd, 0, sizeof(int64_t) * nprof, (cudaStream_t)stream);
+      return cuda_status(e0);
+    }
     return HMG_OK;
   }
   Dev dg(db->device);
@@ -1758,7 +1766,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
       }
       {
         std::vector<Scratch*> SS;
-        struct Bufs { int32_t* surv; int16_t* vraw; void* tmp; };
+        struct Bufs { int32_t* surv; int16_t* vraw; void* tmp; uint8_t* vpass; int32_t* fl; };
         std::vector<Bufs> B;
         hmg_status s = HMG_OK;
         for (int k = 0; k < std::max(ns, 1); ++k) {
@@ -1768,6 +1776,10 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
           b.surv = (int32_t*)SS.back()->get(sizeof(int32_t) * (size_t)n, &e);
           b.vraw = (int16_t*)SS.back()->get(sizeof(int16_t) * (size_t)n, &e);
           b.tmp = SS.back()->get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
+          if (tail->fwd_nats) {
+            b.vpass = (uint8_t*)SS.back()->get((size_t)n, &e);
+            b.fl = (int32_t*)SS.back()->get(sizeof(int32_t) * (size_t)n, &e);
+          }
           B.push_back(b);
         }
         for (int r = 0; r < nprof && !e && s == HMG_OK; ++r) {
@@ -1781,8 +1793,15 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
           if (e) break;
           s = run_vit(pi, db, B[k].surv, tail->n_survivors + i, sk, B[k].vraw, *SS[k], nullptr, 0, false, n);
           if (s != HMG_OK) break;
+          if (tail->fwd_nats && (e = cudaMemsetAsync(B[k].vpass, 0, (size_t)n, sk))) break;
           e = vit_finish(B[k].vraw, B[k].surv, tail->n_survivors + i, n, db->d_len, db->d_order, tv[r],
-                         tail->vit_raw + ro, nullptr, tail->flags + ro, sk);
+                         tail->vit_raw + ro, nullptr, tail->flags + ro, sk, tail->fwd_nats ? B[k].vpass : nullptr);
+          if (e || !tail->fwd_nats) continue;
+          // Forward stage on this profile's Viterbi passes (Fig 1)
+          if ((e = compact_flags(B[k].vpass, n, db->d_order, B[k].fl, tail->fwd_ids + ro, tail->n_fwd + i, B[k].tmp,
+                                 sk)))
+            break;
+          s = run_fwd(pi, db, B[k].fl, tail->n_fwd + i, sk, tail->fwd_nats + ro, tail->flags + ro, *SS[k]);
         }
         for (auto* x : SS) delete x;                 // stream-ordered frees on each side stream
         if (s != HMG_OK) return s;
@@ -1810,11 +1829,14 @@ hmg_status hmg_msv_batch(const hmg_profile* const* profs, int nprof, const hmg_d
 
 hmg_status hmg_pipeline_batch(const hmg_profile* const* profs, int nprof, const hmg_db* db, double F1, double F2,
                               void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
-                              int32_t* survivor_ids, int64_t* n_survivors) {
+                              int32_t* survivor_ids, int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids,
+                              int64_t* n_fwd) {
   if (!(F2 > 0.0 && F2 <= 1.0)) return HMG_EINVAL;
   if (db && db->nseq && (!vit_raw || !flags || !survivor_ids || !n_survivors)) return HMG_EINVAL;
   if (db && !db->nseq && !n_survivors) return HMG_EINVAL;
-  BatchTail t{F2, vit_raw, flags, survivor_ids, n_survivors};
+  if ((fwd_nats != nullptr) != (n_fwd != nullptr) || (fwd_nats != nullptr) != (fwd_ids != nullptr))
+    return HMG_EINVAL;
+  BatchTail t{F2, vit_raw, flags, survivor_ids, n_survivors, fwd_nats, fwd_ids, n_fwd};
   return msv_batch_impl(profs, nprof, db, F1, stream, msv_raw, nullptr, &t);
 }
 

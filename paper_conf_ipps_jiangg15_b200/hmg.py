@@ -56,7 +56,7 @@ SIGNATURES = {
     "hmg_forward": (c_int, [c_p, c_p, c_p, c_i64, c_p, c_p]),
     "hmg_pipeline_forward": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_batch": (c_int, [c_p, c_int, c_p, c_d, c_p, c_p, c_p]),
-    "hmg_pipeline_batch": (c_int, [c_p, c_int, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
+    "hmg_pipeline_batch": (c_int, [c_p, c_int, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_nats": (c_f, [c_int, c_int]),
     "hmg_vit_nats": (c_f, [c_int, c_int]),
     "hmg_null1_nats": (c_f, [c_int]),
@@ -280,12 +280,14 @@ def hmg_msv_batch(profiles, db: Database, raw, pass_=None, F1: float = 0.02, str
 
 
 def hmg_pipeline_batch(profiles, db: Database, msv_raw, vit_raw, flags, survivor_ids, n_survivors,
-                       F1: float = 0.02, F2: float = 1e-3, stream=None):
-    """Fig 1 filter pipeline for every profile of a batch (f4); outputs are [nprof][nseq] rows."""
+                       F1: float = 0.02, F2: float = 1e-3, stream=None, fwd_nats=None, fwd_ids=None, n_fwd=None):
+    """Fig 1 filter pipeline for every profile of a batch (f4); outputs are [nprof][nseq] rows;
+    with fwd_nats / fwd_ids / n_fwd also the Forward stage on each profile's Viterbi passes."""
     arr = (c_p * len(profiles))(*[p.handle for p in profiles])
     _check(lib().hmg_pipeline_batch(arr, len(profiles), db.handle, F1, F2, _stream_ptr(stream), _dev_ptr(msv_raw),
                                     _dev_ptr(vit_raw), _dev_ptr(flags), _dev_ptr(survivor_ids),
-                                    _dev_ptr(n_survivors)), "hmg_pipeline_batch")
+                                    _dev_ptr(n_survivors), _dev_ptr(fwd_nats), _dev_ptr(fwd_ids),
+                                    _dev_ptr(n_fwd)), "hmg_pipeline_batch")
 
 
 def alloc_batch_outputs(nprof: int, nseq: int, device: int = 0):
@@ -297,6 +299,15 @@ def alloc_batch_outputs(nprof: int, nseq: int, device: int = 0):
                 flags=torch.zeros((nprof, nseq), dtype=torch.uint8, device=dev),
                 survivor_ids=torch.zeros((nprof, max(nseq, 1)), dtype=torch.int32, device=dev),
                 n_survivors=torch.zeros(nprof, dtype=torch.int64, device=dev))
+
+
+def alloc_batch_forward_outputs(nprof: int, nseq: int, device: int = 0):
+    """Optional Forward outputs of hmg_pipeline_batch."""
+    import torch
+    dev = torch.device("cuda", device)
+    return dict(fwd_nats=torch.full((nprof, nseq), float("nan"), dtype=torch.float32, device=dev),
+                fwd_ids=torch.zeros((nprof, max(nseq, 1)), dtype=torch.int32, device=dev),
+                n_fwd=torch.zeros(nprof, dtype=torch.int64, device=dev))
 
 
 def hmg_msv_nats(raw: int, L: int) -> float:

@@ -146,8 +146,9 @@ def test_batch_invalid_and_empty():
 
 
 def test_pipeline_batch_equals_per_profile_pipelines():
-    """hmg_pipeline_batch (MSV batch -> per-profile compaction + Viterbi on side streams) equals one
-    hmg_pipeline call per profile on every output, and the oracle on the survivors of two rows."""
+    """hmg_pipeline_batch (MSV batch -> per-profile compaction + Viterbi + Forward on side streams)
+    equals one hmg_pipeline_forward call per profile on every output, and the oracle on the
+    survivors of two rows."""
     prof1, dbs = synth.config(1)
     dsq, off = dbs.materialize()
     lam = math.log(2)
@@ -157,12 +158,20 @@ def test_pipeline_batch_equals_per_profile_pipelines():
     P = [hmg.Profile(pr.msc, pr.tsc, ev=ev) for pr, ev in zip(profs, evs)]
     db = hmg.Database(dsq, off)
     out = hmg.alloc_batch_outputs(len(P), db.nseq)
-    hmg.hmg_pipeline_batch(P, db, F1=0.1, F2=0.05, **out)
+    fo = hmg.alloc_batch_forward_outputs(len(P), db.nseq)
+    hmg.hmg_pipeline_batch(P, db, F1=0.1, F2=0.05, **out, **fo)
     torch.cuda.synchronize()
     for i, p in enumerate(P):
         one = hmg.alloc_outputs(db.nseq)
-        hmg.hmg_pipeline(p, db, F1=0.1, F2=0.05, **one)
+        f1 = hmg.alloc_forward_outputs(db.nseq)
+        hmg.hmg_pipeline_forward(p, db, F1=0.1, F2=0.05, **one, **f1)
         torch.cuda.synchronize()
+        nf = int(f1["n_fwd"].item())
+        assert int(fo["n_fwd"][i].item()) == nf
+        assert torch.equal(fo["fwd_ids"][i][:nf], f1["fwd_ids"][:nf])
+        assert torch.equal(fo["fwd_nats"][i].isnan(), f1["fwd_nats"].isnan())
+        fi = f1["fwd_ids"][:nf].long()
+        assert torch.equal(fo["fwd_nats"][i][fi], f1["fwd_nats"][fi])   # same kernel, same inputs
         ns = int(one["n_survivors"].item())
         assert int(out["n_survivors"][i].item()) == ns > 0
         assert torch.equal(out["msv_raw"][i], one["msv_raw"])

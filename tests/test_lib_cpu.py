@@ -162,7 +162,9 @@ def test_host_only_handles_rejected_by_compute_calls(L):
     assert L.hmg_msv_batch(arr, 1, d.handle, 0.02, None, vp(1), None) == hmg.HMG_EINVAL
     assert L.hmg_msv_batch(arr, 0, d.handle, 0.02, None, vp(1), None) == hmg.HMG_EINVAL
     assert L.hmg_pipeline_batch(arr, 1, d.handle, 0.02, 2.0, None, vp(1), vp(1), vp(1), vp(1),
-                                vp(1)) == hmg.HMG_EINVAL
+                                vp(1), None, None, None) == hmg.HMG_EINVAL
+    assert L.hmg_pipeline_batch(arr, 1, d.handle, 0.02, 1e-3, None, vp(1), vp(1), vp(1), vp(1),
+                                vp(1), vp(1), None, None) == hmg.HMG_EINVAL     # Forward outputs: all or none
 
 
 def test_forward_geometry_host_only(L):
