@@ -80,6 +80,8 @@ typedef struct {
                                        or M > 4096) */
   int fwd_rows_smem;                /* emission-odds rows staged in shared memory (the rest via L1) */
   int fwd_seqs_per_block;           /* Forward kernel: sequences per block sharing the staged table */
+  int fwd_lanes;                    /* Forward kernel: threads per sequence (8 = sub-warp lane groups
+                                       for M <= 32; else 32 x fwd_warps) */
 } hmg_quant;
 
 /* ---------------------------------------------------------------- profile */

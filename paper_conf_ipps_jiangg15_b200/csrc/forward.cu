@@ -41,47 +41,61 @@ const void* fwd_ptr_w2(int q, int s);
 const void* fwd_ptr_w4(int q, int s);
 const void* fwd_ptr_w8(int q, int s);
 const void* fwd_ptr_w16(int q, int s);
+const void* fwd_ptr_sub(int gl, int q, int s);
 
-static const void* fwd_fn(int W, int Q, int S) {
-  switch (W) {
-    case 1: return fwd_ptr_w1(Q, S);
-    case 2: return fwd_ptr_w2(Q, S);
-    case 4: return fwd_ptr_w4(Q, S);
-    case 8: return fwd_ptr_w8(Q, S);
-    case 16: return fwd_ptr_w16(Q, S);
+// T = threads per sequence: 8 (sub-warp lane groups) or 32 W.
+static const void* fwd_fn(int T, int Q, int S) {
+  switch (T) {
+    case 8: return fwd_ptr_sub(T, Q, S);
+    case 32: return fwd_ptr_w1(Q, S);
+    case 64: return fwd_ptr_w2(Q, S);
+    case 128: return fwd_ptr_w4(Q, S);
+    case 256: return fwd_ptr_w8(Q, S);
+    case 512: return fwd_ptr_w16(Q, S);
   }
   return nullptr;
 }
 
-static const int kFwdS[][4] = {{2, 4, 8, 12}, {1, 2, 4, 6}, {1, 2, 3, 0}, {1, 0, 0, 0}, {1, 0, 0, 0}};
+static const int* fwd_s_list(int T) {
+  static const int s8[] = {8, 16, 32, 0}, s32[] = {2, 4, 8, 12, 0}, s64[] = {1, 2, 4, 6, 0},
+                   s128[] = {1, 2, 3, 0}, s256[] = {1, 0};
+  switch (T) {
+    case 8: return s8;
+    case 32: return s32;
+    case 64: return s64;
+    case 128: return s128;
+  }
+  return s256;
+}
 
-static size_t fwd_group_floats(int W) { return (size_t)2 * ((7 * W + 3) / 4 * 4) + 4; }   // forward.cuh
+static size_t fwd_group_floats(int T) {        // forward.cuh: 2 parity buffers + slot
+  const int W = T >= 32 ? T / 32 : 1;
+  return (size_t)2 * ((7 * W + 3) / 4 * 4) + 4;
+}
 
-size_t fwd_smem(int W, int Q, int rows, int S) {
-  return ((size_t)rows * 32 * W * Q + (size_t)S * fwd_group_floats(W)) * sizeof(float);
+size_t fwd_smem(int T, int Q, int rows, int S) {
+  return ((size_t)rows * T * Q + (size_t)S * fwd_group_floats(T)) * sizeof(float);
 }
 
 // Sequences per block: the instantiated S with the most resident warps per SM (registers and the
 // shared emission table decide), the smaller S on ties (finer work granularity).
-int fwd_pick_s(int W, int Q, int rows) {
-  const int wi = W == 1 ? 0 : W == 2 ? 1 : W == 4 ? 2 : W == 8 ? 3 : 4;
+int fwd_pick_s(int T, int Q, int rows) {
   int best = 0, bw = 0;
-  for (int i = 0; i < 4; ++i) {
-    const int S = kFwdS[wi][i];
-    if (S == 0) break;
-    const void* fn = fwd_fn(W, Q, S);
+  for (const int* ps = fwd_s_list(T); *ps; ++ps) {
+    const int S = *ps;
+    const void* fn = fwd_fn(T, Q, S);
     if (!fn) continue;
-    const size_t smem = fwd_smem(W, Q, rows, S);
+    const size_t smem = fwd_smem(T, Q, rows, S);
     if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
       cudaGetLastError();
       continue;
     }
     int per = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, 32 * W * S, smem) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, T * S, smem) != cudaSuccess) {
       cudaGetLastError();
       continue;
     }
-    const int warps = per * W * S;
+    const int warps = per * T * S / 32;
     if (warps > bw) {
       bw = warps;
       best = S;
@@ -90,25 +104,33 @@ int fwd_pick_s(int W, int Q, int rows) {
   return best;
 }
 
-// Geometry: the fewest warps per sequence at qmax nodes per thread (16 for the lean variant, up
-// to 8 warps; else 8, up to 16 warps), then the fewest nodes per thread (2, 4, 8, 16) for that
-// width; models above 4096 nodes are not supported by this kernel.
-bool fwd_geometry(int M, int* W, int* Q, int qmax) {
+// Geometry (T threads per sequence, Q nodes per thread): models up to 32 nodes take sub-warp
+// groups of 8 lanes (4 sequences per warp, SURVEY 7 hard part 5: at M = 64-128 the 8/16-lane
+// groups with 8 nodes per thread measured 10% slower than a warp with 2-4 nodes, whose lower
+// register count doubles the resident warps); above,
+// the fewest warps at qmax nodes per thread (16 for the lean variant, up to 8 warps; else 8, up
+// to 16 warps), then the fewest nodes per thread for that width; above 4096 nodes: none.
+bool fwd_geometry(int M, int* T, int* Q, int qmax) {
+  if (M <= 32) {                       // measured: only tiny models gain (profiles/fwd_bench_r01f.jsonl)
+    *T = 8;
+    *Q = M <= 16 ? 2 : 4;
+    return true;
+  }
   const int wmax = qmax >= 16 ? 8 : 16;   // 16 nodes/thread: <= 256 threads per sequence (registers)
   int w = 1;
   while (32 * w * qmax < M && w < wmax) w *= 2;
   if (32 * w * qmax < M) return false;
   int q = 2;
   while (32 * w * q < M) q *= 2;
-  *W = w;
+  *T = 32 * w;
   *Q = q;
   return true;
 }
 
 // Host tables (odds, float32) in the kernel's layouts.  msc: [M][29] nats, tsc: [M][8] nats.
-void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
+void fwd_tables(int M, int T, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
                 std::vector<float>* tr, std::vector<float>* cst) {
-  const int T = 32 * W, V = Q >= 4 ? 4 : Q, C = Q / V, ROWF = T * Q;
+  const int V = Q >= 4 ? 4 : Q, C = Q / V, ROWF = T * Q, SEG = T < 32 ? T : 32;   // SEG: shuffle segment
   etab->assign((size_t)kRows * ROWF, 0.0f);
   for (int x = 0; x < kAlpha; ++x)
     for (int t = 0; t < T; ++t)
@@ -141,12 +163,13 @@ void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::ve
   cst->assign((size_t)(kFwdConst + Q) * T, 0.0f);
   auto C_ = [&](int i, int t) -> float& { return (*cst)[(size_t)i * T + t]; };
   for (int t = 0; t < T; ++t) {
-    const int ws = t & ~31, lane = t & 31;
-    for (int d = 0; d < 5; ++d) C_(d, t) = lane >= (1 << d) ? (float)slope(t - (1 << d) + 1, t) : 0.0f;
+    const int ws = t & ~(SEG - 1), lane = t & (SEG - 1);
+    for (int d = 0; d < 5; ++d)
+      C_(d, t) = (1 << d) < SEG && lane >= (1 << d) ? (float)slope(t - (1 << d) + 1, t) : 0.0f;
     C_(5, t) = (float)slope(ws, t - 1);
     C_(6, t) = (float)slope(ws, t);
     double g = 0.0, run = 1.0;          // G_t = sum_{t'>t} Ps(t') prod_{t<m<t'} A_m
-    for (int u = t + 1; u < T; ++u) {
+    for (int u = t + 1; u < T; ++u) {   // (over the whole sequence's threads)
       g += Ps[u] * run;
       run *= A[u];
     }
@@ -156,14 +179,14 @@ void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::ve
   }
 }
 
-cudaError_t launch_fwd(int W, int Q, int S, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok) {
-  const void* fn = fwd_fn(W, Q, S);
+cudaError_t launch_fwd(int T, int Q, int S, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok) {
+  const void* fn = fwd_fn(T, Q, S);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
-  const size_t smem = fwd_smem(W, Q, rows_smem, S);
+  const size_t smem = fwd_smem(T, Q, rows_smem, S);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int BT = 32 * W * S;
+  const int BT = T * S;
   int dev = 0, nsm = 0, per = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);

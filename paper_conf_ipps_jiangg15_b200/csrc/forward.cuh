@@ -28,17 +28,23 @@ __device__ __forceinline__ void group_sync(int id, int nthreads) {
 //   9..   P_q     prod_{q'<q} tDD_{q'} within the thread (D_q = Dloc_q + c_in P_q)
 constexpr int kFwdConst = 9;
 
-template <int W, int Q, int S>
-__global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
-  constexpr int T = 32 * W;                    // threads per sequence
+// GL < 32 (W = 1 only): a sequence takes a group of GL lanes and a warp scores 32 / GL sequences of
+// adjacent length rank in lockstep, iterating to the longest of them (rows past a sequence's end
+// leave its special states untouched); shuffles run within the GL-lane segments.
+template <int W, int Q, int S, int GL = 32>
+__global__ void __launch_bounds__((W == 1 ? GL : 32 * W) * S, 1) fwd_kernel(const FwdArgs a) {
+  static_assert(GL == 32 || W == 1, "lane groups below a warp need W = 1");
+  constexpr int T = W == 1 ? GL : 32 * W;      // threads per sequence
   constexpr int BT = T * S;                    // threads per block (S sequences)
+  constexpr int NGW = 32 / T > 0 ? 32 / T : 1; // sequences per warp
+  constexpr int LG = GL == 8 ? 3 : GL == 16 ? 4 : 5;   // scan / reduction steps
   constexpr int V = FwdVec<Q>::V;              // floats per vector load
   constexpr int C = Q / V;                     // chunks per thread
   constexpr int ROWF = T * Q;                  // floats per residue row
   constexpr int PAR = (7 * W + 3) / 4 * 4;     // floats per parity buffer of a group (16-B aligned)
   extern __shared__ float4 smem4[];
   float* tab = reinterpret_cast<float*>(smem4);                   // [rows_smem][C][T][V]
-  const int g = threadIdx.x / T, t = threadIdx.x % T, w = t >> 5, lane = t & 31;
+  const int g = threadIdx.x / T, t = threadIdx.x % T, w = t >> 5, lane = t & (GL - 1);
   float* grp = tab + (size_t)a.rows_smem * ROWF + (size_t)g * (2 * PAR + 4);
   int* slot = reinterpret_cast<int*>(grp + 2 * PAR);
   const int bar = 1 + g;
@@ -63,9 +69,9 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
   }
   if constexpr (LEAN) P[0] = a.cst[(kFwdConst + Q / 2) * T + t];   // P_{Q/2}
   const float PL = a.cst[(kFwdConst + Q - 1) * T + t];             // P_{Q-1} (cross-warp carry)
-  float mul[5];
+  float mul[LG];
 #pragma unroll
-  for (int d = 0; d < 5; ++d) mul[d] = a.cst[d * T + t];
+  for (int d = 0; d < LG; ++d) mul[d] = a.cst[d * T + t];
   const float pa = a.cst[5 * T + t], ai = a.cst[6 * T + t], G = a.cst[7 * T + t], paP = a.cst[8 * T + t];
   __syncthreads();
 
@@ -73,22 +79,28 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
   int par = 0;
   for (;;) {
     int64_t idx;
-    if constexpr (W == 1) {
+    if constexpr (W == 1) {                    // one fetch per warp: NGW adjacent sequences
       unsigned long long v = 0;
-      if (lane == 0) v = atomicAdd(a.counter, 1ull);
+      if ((threadIdx.x & 31) == 0) v = atomicAdd(a.counter, (unsigned long long)NGW);
       idx = (int64_t)__shfl_sync(0xffffffffu, v, 0);
+      if (idx >= n) break;
+      idx += (threadIdx.x & 31) / T;
     } else {
       if (t == 0) *slot = (int)atomicAdd(a.counter, 1ull);
       group_sync(bar, T);
       idx = *slot;
       group_sync(bar, T);
+      if (idx >= n) break;
     }
-    if (idx >= n) break;
-    const int s = a.list ? a.list[idx] : (int)idx;
-    const int L = a.len[s];
-    const uint32_t* wp = a.words + (size_t)a.woff16[s] * 4;
-    const float loop = (float)((double)L / (double)(L + 3));
-    const float move = (float)(3.0 / (double)(L + 3));
+    const bool valid = idx < n;
+    const int s = valid ? (a.list ? a.list[idx] : (int)idx) : 0;
+    const int L = valid ? a.len[s] : 0;
+    int Lw = L;                                // rows the warp iterates: its longest sequence
+#pragma unroll
+    for (int o = 16; o >= T; o >>= 1) Lw = max(Lw, __shfl_xor_sync(0xffffffffu, Lw, o));
+    const uint32_t* wp = a.words + (size_t)(valid ? a.woff16[s] : 0) * 4;
+    const float loop = valid ? (float)((double)L / (double)(L + 3)) : 0.0f;
+    const float move = valid ? (float)(3.0 / (double)(L + 3)) : 0.0f;
     float Mc[Q], Ic[Q], Dc[Q], e[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) Mc[q] = Ic[q] = Dc[q] = 0.0f;
@@ -109,24 +121,26 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
         }
       }
     };
-    const int nw = (L + 5) / 6;
-    for (int w0 = 0; w0 < nw; w0 += 32) {
+    const int nw = (L + 5) / 6, nww = (Lw + 5) / 6;
+    for (int w0 = 0; w0 < nww; w0 += GL) {
       const uint32_t wreg = (w0 + lane < nw) ? __ldg(wp + w0 + lane) : 0u;
-      const int wend = min(32, nw - w0);
+      const int wend = min(GL, nww - w0);
 #pragma unroll 1
       for (int j = 0; j < wend; ++j) {
-        const uint32_t word = __shfl_sync(0xffffffffu, wreg, j);
-        const int bend = min(6, L - 6 * (w0 + j));
+        const uint32_t word = __shfl_sync(0xffffffffu, wreg, j, GL);
+        const int bend = min(6, Lw - 6 * (w0 + j));
 #pragma unroll 1
         for (int b = 0; b < bend; ++b) {
-          const int x = (word >> (5 * b)) & 31;
+          // rows past the sequence's end (lane groups only): cells only, specials frozen
+          const bool act = T >= 32 || 6 * (w0 + j) + b < L;
+          const int x = act ? (int)((word >> (5 * b)) & 31) : 0;
           // x is uniform over the group (>= one warp): shared-memory rows by LDS, the rest via L1
           if (x < a.rows_smem) load_row(tab + (size_t)x * ROWF, true);
           else load_row(a.etab + (size_t)x * ROWF, false);
           // diagonal carries: row i-1 cells of node t Q (thread t-1)
-          float cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1);
-          float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1);
-          float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1);
+          float cM = __shfl_up_sync(0xffffffffu, Mc[Q - 1], 1, GL);
+          float cI = __shfl_up_sync(0xffffffffu, Ic[Q - 1], 1, GL);
+          float cD = __shfl_up_sync(0xffffffffu, Dc[Q - 1], 1, GL);
           if (lane == 0) { cM = nM; cI = nI; cD = nD; }
           // M and I from row i-1 (descending q: index q-1 still holds row i-1)
 #pragma unroll
@@ -153,12 +167,12 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
           // scan of the chain outputs (constant slopes) and the E reduction, independent chains
           float ib = bsum;
 #pragma unroll
-          for (int d = 0; d < 5; ++d) {
-            const float ub = __shfl_up_sync(0xffffffffu, ib, 1 << d);
-            econ += __shfl_xor_sync(0xffffffffu, econ, 16 >> d);
+          for (int d = 0; d < LG; ++d) {
+            const float ub = __shfl_up_sync(0xffffffffu, ib, 1 << d, GL);
+            econ += __shfl_xor_sync(0xffffffffu, econ, (GL / 2) >> d);
             if (lane >= (1 << d)) ib = fmaf(mul[d], ub, ib);
           }
-          const float pb = __shfl_up_sync(0xffffffffu, ib, 1);
+          const float pb = __shfl_up_sync(0xffffffffu, ib, 1, GL);
           float xE = econ, cw = 0.0f;
           if constexpr (W > 1) {
             float* buf = grp + par * PAR;
@@ -201,7 +215,8 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
 #pragma unroll
             for (int q = 0; q < Q; ++q) Dc[q] = fmaf(cin, P[q], Dc[q]);
           }
-          // specials (every thread, identical values)
+          // specials (every thread of the group, identical values; frozen past the sequence's end)
+          if (T < 32 && !act) continue;
           xN *= loop;
           xJ = fmaf(xJ, loop, 0.5f * xE);
           xC = fmaf(xC, loop, 0.5f * xE);
@@ -218,7 +233,7 @@ __global__ void __launch_bounds__(32 * W * S, 1) fwd_kernel(const FwdArgs a) {
         }
       }
     }
-    if (t == 0) {
+    if (t == 0 && valid) {
       const double sc = (double)xC * (double)move;
       const int c = a.order[s];
       a.out[c] = sc > 0.0 ? (float)(log(sc) + (double)scale_exp * 0.6931471805599453) : -INFINITY;

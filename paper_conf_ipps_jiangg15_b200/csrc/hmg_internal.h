@@ -165,6 +165,7 @@ struct hmg_profile {
   int32_t* d_long_tr = nullptr;
   // Forward stage (forward.cu): fwd_kernel<fwd_W, fwd_Q>, emission rows x < fwd_rows in shared memory
   int fwd_W = 0, fwd_Q = 0, fwd_rows = 0, fwd_S = 1;   // S sequences per block
+  int fwd_T = 0;                    // threads per sequence (8 or 32 fwd_W)
   float msc_max = 0.f;              // largest emission log-odds (odds-space range check)
   float* d_fwd_e = nullptr;         // emission odds [kRows][C][T][V]
   float* d_fwd_t = nullptr;         // transition odds [8][T][Q]
@@ -250,12 +251,13 @@ cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* 
                           int32_t* ids_caller, int64_t* count, void* tmp, cudaStream_t st);
 
 // Forward stage (forward.cu)
-bool fwd_geometry(int M, int* W, int* Q, int qmax);
-size_t fwd_smem(int W, int Q, int rows, int S);
-int fwd_pick_s(int W, int Q, int rows);
-void fwd_tables(int M, int W, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
+// T = threads per sequence (8: sub-warp lane groups; 32 W: W warps)
+bool fwd_geometry(int M, int* T, int* Q, int qmax);
+size_t fwd_smem(int T, int Q, int rows, int S);
+int fwd_pick_s(int T, int Q, int rows);
+void fwd_tables(int M, int T, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
                 std::vector<float>* tr, std::vector<float>* cst);
-cudaError_t launch_fwd(int W, int Q, int S, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_fwd(int T, int Q, int S, int rows_smem, const FwdArgs& a, cudaStream_t st, int* ok);
 cudaError_t to_sorted_ids(const int32_t* caller_ids, int64_t n, const int32_t* inv_order, int32_t* sorted_ids,
                           cudaStream_t st);
 cudaError_t set_count(int64_t* d, int64_t v, cudaStream_t st);

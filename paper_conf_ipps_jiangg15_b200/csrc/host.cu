@@ -780,13 +780,13 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   for (size_t i = 0; i < (size_t)M * kAlpha; ++i) p->msc_max = std::max(p->msc_max, msc[i]);
   // ---- Forward stage geometry (forward.cu): emission rows staged in shared memory as fit
   const int fwd_qmax = env_int("HMG_FWD_QMAX", 16) >= 16 ? 16 : 8;   // 16: profiles/fwd_bench_r01e.jsonl
-  if (tsc && (fwd_geometry(M, &p->fwd_W, &p->fwd_Q, fwd_qmax) || fwd_geometry(M, &p->fwd_W, &p->fwd_Q, 8))) {
-    const int wo = env_int("HMG_FWD_W", 0);   // wider groups (shorter rows, more threads per sequence)
+  if (tsc && (fwd_geometry(M, &p->fwd_T, &p->fwd_Q, fwd_qmax) || fwd_geometry(M, &p->fwd_T, &p->fwd_Q, 8))) {
+    const int wo = env_int("HMG_FWD_W", 0);   // whole warps per sequence (1 = no sub-warp groups)
     if (wo == 1 || wo == 2 || wo == 4 || wo == 8 || wo == 16) {
       int q = 2;
       while (32 * wo * q < M && q < 16) q *= 2;
       if (32 * wo * q >= M) {
-        p->fwd_W = wo;
+        p->fwd_T = 32 * wo;
         p->fwd_Q = q;
       }
     }
@@ -794,14 +794,15 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     if (device >= 0) cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
     else smax = 227 * 1024;
     int rows = kAlpha;
-    while (rows > 0 && fwd_smem(p->fwd_W, p->fwd_Q, rows, 1) > (size_t)smax) --rows;
+    while (rows > 0 && fwd_smem(p->fwd_T, p->fwd_Q, rows, 1) > (size_t)smax) --rows;
     p->fwd_rows = rows;
+    p->fwd_W = p->fwd_T >= 32 ? p->fwd_T / 32 : 1;
     if (device >= 0) {
       Dev dg(device);
-      p->fwd_S = fwd_pick_s(p->fwd_W, p->fwd_Q, rows);
+      p->fwd_S = fwd_pick_s(p->fwd_T, p->fwd_Q, rows);
       const int so = env_int("HMG_FWD_S", 0);
       if (so > 0) p->fwd_S = so;
-      if (p->fwd_S == 0) p->fwd_W = 0;   // no launchable configuration: Forward unsupported
+      if (p->fwd_S == 0) p->fwd_W = p->fwd_T = 0;   // no launchable configuration: Forward unsupported
     }
   }
   // ---- kernel geometry and device tables
@@ -963,7 +964,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   }
   if (st == HMG_OK && p->fwd_W > 0) {
     std::vector<float> e, t, c;
-    fwd_tables(M, p->fwd_W, p->fwd_Q, msc, tsc, &e, &t, &c);
+    fwd_tables(M, p->fwd_T, p->fwd_Q, msc, tsc, &e, &t, &c);
     st = upload(&p->d_fwd_e, e.data(), e.size());
     if (st == HMG_OK) st = upload(&p->d_fwd_t, t.data(), t.size());
     if (st == HMG_OK) st = upload(&p->d_fwd_c, c.data(), c.size());
@@ -1062,6 +1063,7 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->vit_pair_lanes = p->pair_G;
   q->vit_pair_regs = p->pair_Q;
   q->fwd_warps = p->fwd_W;
+  q->fwd_lanes = p->fwd_T;
   q->fwd_nodes = p->fwd_Q;
   q->fwd_rows_smem = p->fwd_rows;
   q->fwd_seqs_per_block = p->fwd_S;
@@ -1435,7 +1437,7 @@ static hmg_status run_fwd(const hmg_profile* p, const hmg_db* db, const int32_t*
   a.flags = flags;
   a.counter = ctr;
   int ok = 0;
-  if ((e = launch_fwd(p->fwd_W, p->fwd_Q, p->fwd_S, p->fwd_rows, a, st, &ok))) return cuda_status(e);
+  if ((e = launch_fwd(p->fwd_T, p->fwd_Q, p->fwd_S, p->fwd_rows, a, st, &ok))) return cuda_status(e);
   return ok ? HMG_OK : HMG_EUNSUPPORTED;
 }
 

@@ -97,7 +97,7 @@ def test_fwd_model_lengths(M, dd):
     dsq, off = _ragged(rng, n=n, lmax=300 if M > 1500 else 500)
     got, p = _fwd_gpu(prof.msc, prof.tsc, dsq, off)
     q = p.quant()
-    assert q["fwd_warps"] * 32 * q["fwd_nodes"] >= M
+    assert q["fwd_lanes"] * q["fwd_nodes"] >= M
     want = oracle.fwd_db(prof.msc, prof.tsc, dsq, off)
     _assert_close(got, want, np.diff(off), M)
 
@@ -227,8 +227,10 @@ def test_pipeline_forward_config3_full_size():
     assert nf >= 400
 
 
-@pytest.mark.parametrize("M,S,qmax", [(40, 2, 16), (40, 4, 16), (40, 8, 16), (40, 12, 16), (200, 2, 16),
-                                      (200, 12, 16), (300, 1, 8), (300, 2, 8), (300, 4, 8), (300, 6, 8),
+@pytest.mark.parametrize("M,S,qmax", [(10, 4, 16), (10, 32, 16), (30, 8, 16), (30, 16, 16), (32, 32, 16),
+                                      (40, 2, 16), (40, 4, 16), (40, 8, 16), (40, 12, 16), (100, 2, 16),
+                                      (128, 12, 16), (200, 2, 16),
+                                      (200, 12, 16), (200, 4, 16), (300, 1, 8), (300, 2, 8), (300, 4, 8), (300, 6, 8),
                                       (700, 1, 8), (700, 2, 8), (700, 3, 8), (300, 2, 16), (300, 4, 16),
                                       (300, 8, 16), (700, 1, 16), (700, 2, 16), (700, 4, 16)])
 def test_fwd_every_block_shape(M, S, qmax, monkeypatch):

@@ -153,7 +153,7 @@ def test_host_only_handles_rejected_by_compute_calls(L):
     p = hmg.Profile(msc, tsc, device=-1)
     d = hmg.Database(np.zeros(12, np.uint8), np.array([0, 5, 12]), device=-1)
     q = p.quant()
-    assert q["fwd_warps"] == 1 and q["fwd_nodes"] == 2 and q["fwd_rows_smem"] == 29
+    assert q["fwd_lanes"] == 8 and q["fwd_nodes"] == 2 and q["fwd_rows_smem"] == 29
     vp = ctypes.c_void_p
     assert L.hmg_forward(p.handle, d.handle, None, 0, None, vp(1)) == hmg.HMG_EINVAL
     assert L.hmg_pipeline_forward(p.handle, d.handle, 0.02, 1e-3, None, vp(1), vp(1), vp(1), vp(1), vp(1),
@@ -168,12 +168,14 @@ def test_host_only_handles_rejected_by_compute_calls(L):
 
 
 def test_forward_geometry_host_only(L):
-    """Forward kernel geometry: fewest warps at 16 nodes per thread, then fewest
-    nodes; unsupported above 4096 nodes."""
-    for M, (W, Qn) in {1: (1, 2), 64: (1, 2), 65: (1, 4), 129: (1, 8), 256: (1, 8), 257: (1, 16),
-                       400: (1, 16), 513: (2, 16), 1000: (2, 16), 2048: (4, 16), 4096: (8, 16)}.items():
+    """Forward kernel geometry: 8-lane groups up to M = 32, then the
+    fewest warps at 16 nodes per thread and the fewest nodes; unsupported above 4096 nodes."""
+    for M, (T, Qn) in {1: (8, 2), 16: (8, 2), 17: (8, 4), 32: (8, 4), 33: (32, 2), 64: (32, 2), 65: (32, 4),
+                       128: (32, 4), 129: (32, 8),
+                       256: (32, 8), 257: (32, 16), 400: (32, 16), 513: (64, 16), 1000: (64, 16), 2048: (128, 16),
+                       4096: (256, 16)}.items():
         p = hmg.Profile(np.zeros((M, 29), np.float32), np.full((M, 8), -1.0, np.float32), device=-1)
         q = p.quant()
-        assert (q["fwd_warps"], q["fwd_nodes"]) == (W, Qn), M
+        assert (q["fwd_lanes"], q["fwd_nodes"], q["fwd_warps"]) == (T, Qn, max(1, T // 32)), M
     p = hmg.Profile(np.zeros((4097, 29), np.float32), np.full((4097, 8), -1.0, np.float32), device=-1)
     assert p.quant()["fwd_warps"] == 0
