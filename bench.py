@@ -445,8 +445,8 @@ def main():
         e_ms = []
 
         def e2e_step(st):
-            D.upload(img, stream=st)                                       # H2D of the packed DB
-            hmg.hmg_pipeline(P, D, F1=args.F1, F2=args.F2, stream=st, **out)
+            # H2D of the packed DB in 4 length-ordered parts overlapped with the filter
+            hmg.hmg_pipeline_upload(P, D, img, F1=args.F1, F2=args.F2, stream=st, **out)
             h_msv.copy_(out["msv_raw"], non_blocking=True)                 # D2H of the results
             h_vit.copy_(out["vit_raw"], non_blocking=True)
             h_flags.copy_(out["flags"], non_blocking=True)

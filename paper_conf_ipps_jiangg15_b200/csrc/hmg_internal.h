@@ -192,6 +192,7 @@ struct hmg_db {
   int64_t nwords = 0;
   std::vector<int32_t> order;      // sorted -> caller
   std::vector<int32_t> len_sorted;
+  std::vector<uint32_t> woff16_h;  // host copy of the word offsets / 4 (overlapped upload parts)
   uint32_t* d_words = nullptr;
   uint32_t* d_woff16 = nullptr;
   int32_t* d_len = nullptr;

@@ -441,11 +441,12 @@ double mean_len(const hmg_db* db) { return db->nseq ? (double)db->residues / (do
 // first pipe_nlong sequences are scored by the pipeline long lane instead.
 hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S,
                         int64_t pipe_nlong, bool pdl = false, bool mark0 = true,
-                        unsigned long long* ctr_zeroed = nullptr) {
+                        unsigned long long* ctr_zeroed = nullptr, int64_t end = -1) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
   a.raw = raw_sorted;
+  if (end >= 0) a.nseq = end;          // sorted range [pipe_nlong, end) only (overlapped upload)
   if (pipe_nlong >= 0) {
     a.nlong = pipe_nlong;
     a.skip_long = 1;
@@ -1142,6 +1143,7 @@ hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, i
     words += ((L + 5) / 6 + 3) / 4 * 4;   // 16-byte aligned runs
   }
   db->nwords = words;
+  db->woff16_h = woff16;
   // pack 6 residues per word, residue j in bits [5j, 5j+5), pad 31 (Fig 6)
   std::vector<uint32_t> img((size_t)std::max<int64_t>(words, 4), 0xffffffffu);
   for (int64_t j = 0; j < nseq; ++j) {
@@ -1329,9 +1331,16 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
   return cuda_status(e);
 }
 
+static cudaStream_t* side_streams(int device);
+
+// h_image (optional): pinned host copy of the packed DB image (hmg_db_image); it is uploaded in
+// kUploadParts length-ordered parts on a side stream while the MSV kernel scores the parts that
+// have landed (one launch per part), so the H2D overlaps the filter.
+constexpr int kUploadParts = 8;     // capacity; parts used: HMG_UPLOAD_PARTS (default 6)
+
 static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
                                 uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
-                                int64_t* n_survivors, uint8_t* vpass_sorted) {
+                                int64_t* n_survivors, uint8_t* vpass_sorted, const uint32_t* h_image = nullptr) {
   hmg_profile* p = const_cast<hmg_profile*>(pc);
   if (!p || !db || !p->has_tsc || !p->has_ev || p->device != db->device || db->device < 0) return HMG_EINVAL;
   if (!(F1 > 0.0 && F1 <= 1.0) || !(F2 > 0.0 && F2 <= 1.0)) return HMG_EINVAL;
@@ -1361,9 +1370,62 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
                            (p->long_pair || (!p->vit_generic && p->vit_W == 0)) &&
                            !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
-    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2, &e);
+    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2 * kUploadParts, &e);
     if (e) return cuda_status(e);
-    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2, st))) return cuda_status(e);
+    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2 * kUploadParts, st))) return cuda_status(e);
+    // overlapped upload: part boundaries (sorted indices) of about equal residues, part 0 >= the
+    // long lane; part k's words are one contiguous run of the image
+    int64_t bnd[kUploadParts + 1] = {0};
+    int nparts = 1;
+    bnd[1] = n;
+    cudaEvent_t up_ev[kUploadParts] = {};
+    cudaStream_t cs = nullptr;
+    if (h_image) {
+      nparts = std::max(2, std::min(kUploadParts, env_int("HMG_UPLOAD_PARTS", 6)));   // profiles/upload_parts_r01.jsonl
+      const int64_t per = (db->residues + nparts - 1) / nparts;
+      int64_t acc = 0, k = 1;
+      for (int64_t j = 0; j < n && k < nparts; ++j) {
+        acc += db->len_sorted[j];
+        if (acc >= per * k && j + 1 >= nlong) bnd[k++] = j + 1;
+      }
+      while (k < nparts) bnd[k++] = n;
+      bnd[nparts] = n;
+      cudaStream_t* side = side_streams(db->device);
+      if (!side) return HMG_ECUDA;
+      cs = side[0];
+      cudaEvent_t fork = nullptr;
+      if ((e = cudaEventCreateWithFlags(&fork, cudaEventDisableTiming))) return cuda_status(e);
+      if ((e = cudaEventRecord(fork, st)) || (e = cudaStreamWaitEvent(cs, fork, 0))) return cuda_status(e);
+      cudaEventDestroy(fork);
+      const int64_t nw_all = std::max<int64_t>(db->nwords, 4);
+      for (int q = 0; q < nparts; ++q) {
+        const int64_t w0 = bnd[q] < n ? (int64_t)db->woff16_h[bnd[q]] * 4 : nw_all;
+        const int64_t w1 = bnd[q + 1] < n ? (int64_t)db->woff16_h[bnd[q + 1]] * 4 : nw_all;
+        if ((e = cudaEventCreateWithFlags(&up_ev[q], cudaEventDisableTiming))) return cuda_status(e);
+        if (w1 > w0 && (e = cudaMemcpyAsync(db->d_words + w0, h_image + w0, (size_t)(w1 - w0) * 4,
+                                            cudaMemcpyHostToDevice, cs)))
+          return cuda_status(e);
+        if ((e = cudaEventRecord(up_ev[q], cs))) return cuda_status(e);
+      }
+      if ((e = cudaStreamWaitEvent(st, up_ev[0], 0))) return cuda_status(e);
+    }
+    // the parts' MSV kernels run on a second side stream (they never read the long lane's
+    // sequences), so the long lane's exclusive-SM Viterbi overlaps all of them
+    cudaStream_t ms = st;
+    cudaEvent_t ms_done = nullptr;
+    const bool overlap = h_image && p->msv_fast && p->msv_Q > 0;
+    if (h_image && !overlap) {                      // exact-kernel profiles: plain upload first
+      for (int q = 1; q < nparts; ++q)
+        if ((e = cudaStreamWaitEvent(st, up_ev[q], 0))) return cuda_status(e);
+    }
+    if (overlap) {
+      ms = side_streams(db->device)[1];
+      cudaEvent_t f2 = nullptr;
+      if ((e = cudaEventCreateWithFlags(&f2, cudaEventDisableTiming))) return cuda_status(e);
+      if ((e = cudaEventRecord(f2, st)) || (e = cudaStreamWaitEvent(ms, f2, 0))) return cuda_status(e);
+      cudaEventDestroy(f2);
+      if ((e = cudaEventCreateWithFlags(&ms_done, cudaEventDisableTiming))) return cuda_status(e);
+    }
     mark(0, st);
     if (nlong > 0) {
       LongArgs la{};
@@ -1388,8 +1450,23 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       if ((e = launch_pipe_long_vit(p->long_QV, p->long_pair, la, nb, st, &ok))) return cuda_status(e);
       if (!ok) return HMG_EUNSUPPORTED;
     }
-    s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV
-    if (s != HMG_OK) return s;
+    if (!overlap) {
+      s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV
+      if (s != HMG_OK) return s;
+    } else {
+      for (int q = 0; q < nparts; ++q) {          // MSV of each part once it has landed
+        if ((e = cudaStreamWaitEvent(ms, up_ev[q], 0))) return cuda_status(e);
+        const int64_t lo = std::max(bnd[q], nlong), hi = bnd[q + 1];
+        if (hi > lo) {
+          s = run_msv_fast(p, db, ms, raw_sorted, S, lo, false, false, mctr + 2 * q, hi);
+          if (s != HMG_OK) return s;
+        }
+      }
+      if ((e = cudaEventRecord(ms_done, ms)) || (e = cudaStreamWaitEvent(st, ms_done, 0))) return cuda_status(e);
+      cudaEventDestroy(ms_done);
+    }
+    if (h_image)
+      for (int q = 0; q < nparts; ++q) cudaEventDestroy(up_ev[q]);
     s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;
     e = msv_finish(raw_sorted, db->d_len, db->d_order, n, tm, msv_raw, flags, surv, n_survivors, survivor_ids, tmp,
@@ -1411,6 +1488,13 @@ hmg_status hmg_pipeline(const hmg_profile* p, const hmg_db* db, double F1, doubl
                         uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
                         int64_t* n_survivors) {
   return pipeline_impl(p, db, F1, F2, stream, msv_raw, vit_raw, flags, survivor_ids, n_survivors, nullptr);
+}
+
+hmg_status hmg_pipeline_upload(const hmg_profile* p, hmg_db* db, const uint32_t* image, double F1, double F2,
+                               void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
+                               int32_t* survivor_ids, int64_t* n_survivors) {
+  if (!db || !image || db->device < 0) return HMG_EINVAL;
+  return pipeline_impl(p, db, F1, F2, stream, msv_raw, vit_raw, flags, survivor_ids, n_survivors, nullptr, image);
 }
 
 // Forward stage over a sorted-order list (device list + device count, nmax = list capacity).

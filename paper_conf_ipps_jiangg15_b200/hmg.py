@@ -53,6 +53,7 @@ SIGNATURES = {
     "hmg_msv": (c_int, [c_p, c_p, c_d, c_p, c_p, c_p]),
     "hmg_viterbi": (c_int, [c_p, c_p, c_p, c_i64, c_d, c_p, c_p, c_p]),
     "hmg_pipeline": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
+    "hmg_pipeline_upload": (c_int, [c_p, c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_forward": (c_int, [c_p, c_p, c_p, c_i64, c_p, c_p]),
     "hmg_pipeline_forward": (c_int, [c_p, c_p, c_d, c_d, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p, c_p]),
     "hmg_msv_batch": (c_int, [c_p, c_int, c_p, c_d, c_p, c_p, c_p]),
@@ -308,6 +309,16 @@ def alloc_batch_forward_outputs(nprof: int, nseq: int, device: int = 0):
     return dict(fwd_nats=torch.full((nprof, nseq), float("nan"), dtype=torch.float32, device=dev),
                 fwd_ids=torch.zeros((nprof, max(nseq, 1)), dtype=torch.int32, device=dev),
                 n_fwd=torch.zeros(nprof, dtype=torch.int64, device=dev))
+
+
+def hmg_pipeline_upload(profile: Profile, db: Database, image, msv_raw, vit_raw, flags, survivor_ids, n_survivors,
+                        F1: float = 0.02, F2: float = 1e-3, stream=None):
+    """Upload of the packed image (pinned host tensor from Database.image) overlapped with the
+    pipeline: MSV scores each length-ordered part as it lands (hmg_pipeline_upload)."""
+    ptr = c_p(image.data_ptr()) if hasattr(image, "data_ptr") else _np_ptr(image)
+    _check(lib().hmg_pipeline_upload(profile.handle, db.handle, ptr, F1, F2, _stream_ptr(stream),
+                                     _dev_ptr(msv_raw), _dev_ptr(vit_raw), _dev_ptr(flags),
+                                     _dev_ptr(survivor_ids), _dev_ptr(n_survivors)), "hmg_pipeline_upload")
 
 
 def hmg_msv_nats(raw: int, L: int) -> float:

@@ -573,3 +573,30 @@ def test_vit_pair_maxplus_scan(M, monkeypatch):
     dsq, off = _db_from(seqs)
     got, _ = _vit_gpu(msc, tsc, dsq, off)
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
+
+
+@pytest.mark.parametrize("cfg", [1, 3])
+def test_pipeline_upload_overlapped_equals_pipeline(cfg):
+    """hmg_pipeline_upload (packed image re-sent from pinned host memory in 4 length-ordered parts,
+    MSV per part as it lands, long lane alongside) gives hmg_pipeline's outputs exactly; the device
+    image is scrubbed first so every residue read must come from this call's upload."""
+    prof, db = synth.config(cfg)
+    dsq, off = db.materialize()
+    ev = _calibrate(prof) if cfg == 1 else (-9.5, math.log(2), -9.0, math.log(2))
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    D = hmg.Database(dsq, off)
+    ref = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline(p, D, **ref)
+    img = torch.empty(D.packed_bytes // 4, dtype=torch.int32, pin_memory=True)
+    D.image(img)
+    D.upload(torch.zeros_like(img).pin_memory())          # scrub the device copy
+    out = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline_upload(p, D, img, **out)
+    torch.cuda.synchronize()
+    ns = int(ref["n_survivors"].item())
+    assert int(out["n_survivors"].item()) == ns
+    for k in ("msv_raw", "flags"):
+        assert torch.equal(out[k], ref[k]), k
+    assert torch.equal(out["survivor_ids"][:ns], ref["survivor_ids"][:ns])
+    sv = ref["survivor_ids"][:ns].long()
+    assert torch.equal(out["vit_raw"][sv], ref["vit_raw"][sv])
