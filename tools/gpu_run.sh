@@ -18,7 +18,7 @@ B="python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-graph"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv \
   python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --no-graph --batch 0 --no-forward \
   > $O/ncu_launch_bench_$TAG.log 2>&1
-for K in msv_fast vit_pair pipe_long_msv pipe_long_vit; do
+for K in msv_fast vit_pair pipe_long_msv pipe_long_vp; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$K -s 3 -c 1 \
     -o $O/${K}_$TAG -f $B --batch 0 --no-forward > $O/ncu_full_${K}_$TAG.log 2>&1
 done
