@@ -600,3 +600,40 @@ def test_pipeline_upload_overlapped_equals_pipeline(cfg):
     assert torch.equal(out["survivor_ids"][:ns], ref["survivor_ids"][:ns])
     sv = ref["survivor_ids"][:ns].long()
     assert torch.equal(out["vit_raw"][sv], ref["vit_raw"][sv])
+
+
+def test_pipeline_in_cuda_graph():
+    """The bench replays hmg_pipeline (and hmg_pipeline_upload) from a CUDA graph captured once:
+    replays give the eager call's outputs exactly (scratch allocations, memsets, the long lane's
+    programmatic launch and the side-stream upload are all capturable)."""
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    rng = np.random.default_rng(8)
+    extra = [synth.random_dsq(rng, L, 20) for L in (3000, 4100, 5200)]          # long-lane sequences
+    dsq2, off2 = _db_from([dsq[off[i]:off[i + 1]] for i in range(len(off) - 1)] + extra)
+    ev = _calibrate(prof)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    D = hmg.Database(dsq2, off2)
+    assert D.long_lane()[0] >= 3
+    ref = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline(p, D, F1=0.3, F2=0.3, **ref)
+    torch.cuda.synchronize()
+    img = torch.empty(D.packed_bytes // 4, dtype=torch.int32, pin_memory=True)
+    D.image(img)
+    for upload in (False, True):
+        out = hmg.alloc_outputs(D.nseq)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, capture_error_mode="thread_local"):
+            if upload:
+                hmg.hmg_pipeline_upload(p, D, img, F1=0.3, F2=0.3, stream=torch.cuda.current_stream(), **out)
+            else:
+                hmg.hmg_pipeline(p, D, F1=0.3, F2=0.3, stream=torch.cuda.current_stream(), **out)
+        for _ in range(2):
+            g.replay()
+        torch.cuda.synchronize()
+        ns = int(ref["n_survivors"].item())
+        assert int(out["n_survivors"].item()) == ns
+        assert torch.equal(out["msv_raw"], ref["msv_raw"]) and torch.equal(out["flags"], ref["flags"])
+        sv = ref["survivor_ids"][:ns].long()
+        assert torch.equal(out["survivor_ids"][:ns], ref["survivor_ids"][:ns])
+        assert torch.equal(out["vit_raw"][sv], ref["vit_raw"][sv])
