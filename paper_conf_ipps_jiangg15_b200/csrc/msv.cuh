@@ -290,8 +290,20 @@ struct MsvLong {
   static constexpr int QL = (G == 32) ? 0 : (G * Q + 31) / 32;
 };
 
+// Minimum resident blocks per SM for a lane geometry: forcing 3 (<= 85 registers) lets a third
+// 256-thread block share the SM where the measured sweep gains (profiles/msv_minb_r01.jsonl:
+// G = 8, Q = 26: -7%; G = 16, Q = 16: -15%; G = 32, Q = 24 at 2 blocks: -6%); 0 = no bound.
 template <int G, int Q>
-__global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
+constexpr int msv_min_blocks() {
+  if (G == 4 && Q >= 8 && Q <= 10) return 3;
+  if (G == 8 && Q >= 24) return 3;
+  if (G == 16 && Q >= 14 && Q <= 18) return 3;
+  if (G == 32 && Q >= 22 && Q <= 26) return 2;
+  return 0;
+}
+
+template <int G, int Q>
+__device__ __forceinline__ void msv_fast_body(const MsvArgs& a) {
   extern __shared__ uint4 smem4[];
   constexpr int QL = MsvLong<G, Q>::QL;
   constexpr int W0 = MsvLayout<G, Q>::WORDS;   // words of the main table (all copies)
@@ -322,6 +334,20 @@ __global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) {
     if (first + (long long)b >= a.nseq) break;
     msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
   }
+}
+
+template <int G, int Q>
+__global__ void __launch_bounds__(256) msv_fast_kernel(const MsvArgs a) { msv_fast_body<G, Q>(a); }
+
+template <int G, int Q, int MB>
+__global__ void __launch_bounds__(256, MB) msv_fast_kernel_mb(const MsvArgs a) { msv_fast_body<G, Q>(a); }
+
+// the kernel instantiated for (G, Q): with a minimum-blocks bound where it measured faster
+template <int G, int Q>
+const void* msv_fast_entry() {
+  constexpr int MB = msv_min_blocks<G, Q>();
+  if constexpr (MB > 0) return reinterpret_cast<const void*>(&msv_fast_kernel_mb<G, Q, MB>);
+  else return reinterpret_cast<const void*>(&msv_fast_kernel<G, Q>);
 }
 
 }  // namespace hmg

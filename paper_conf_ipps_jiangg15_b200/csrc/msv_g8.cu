@@ -8,7 +8,7 @@ const void* pick(int q) {
   if constexpr (Q > 32) {
     return nullptr;
   } else {
-    if (q == Q) return reinterpret_cast<const void*>(&msv_fast_kernel<8, Q>);
+    if (q == Q) return msv_fast_entry<8, Q>();
     return pick<Q + 1>(q);
   }
 }
