@@ -274,6 +274,8 @@ struct VitPairLane {
   }
 };
 
+// (a register cap for more resident warps -- 96 / 80 / 64 registers -- measured 13% / 77% / 200%
+//  slower on the config-3 Viterbi stage: the row state spills; profiles/vit_minb_r01.jsonl)
 template <int G, int Q, bool SCAN = false>
 __global__ void __launch_bounds__(128) vit_pair_kernel(const VitArgs a) {
   constexpr int ROWW = Q * G;              // s16x2 words per residue row
