@@ -17,7 +17,7 @@ const void* pick_multi(int q) {
   if constexpr (Q > 32) {
     return nullptr;
   } else {
-    if (q == Q) return reinterpret_cast<const void*>(&msv_multi_kernel<8, Q>);
+    if (q == Q) return msv_multi_entry<8, Q>();
     return pick_multi<Q + 1>(q);
   }
 }

@@ -16,7 +16,7 @@
 namespace hmg {
 
 template <int G, int Q>
-__global__ void __launch_bounds__(256) msv_multi_kernel(const MsvMultiArgs m) {
+__device__ __forceinline__ void msv_multi_body(const MsvMultiArgs& m) {
   extern __shared__ uint4 smem4[];
   __shared__ long long item_sh;
   __shared__ unsigned sub_ctr;
@@ -55,6 +55,20 @@ __global__ void __launch_bounds__(256) msv_multi_kernel(const MsvMultiArgs m) {
       msv_batch<G, Q>(a, sm, lo + (long long)b, hi);
     }
   }
+}
+
+template <int G, int Q>
+__global__ void __launch_bounds__(256) msv_multi_kernel(const MsvMultiArgs m) { msv_multi_body<G, Q>(m); }
+
+template <int G, int Q, int MB>
+__global__ void __launch_bounds__(256, MB) msv_multi_kernel_mb(const MsvMultiArgs m) { msv_multi_body<G, Q>(m); }
+
+// the same per-geometry minimum-blocks policy as the single-profile kernel (msv_min_blocks)
+template <int G, int Q>
+const void* msv_multi_entry() {
+  constexpr int MB = msv_min_blocks<G, Q>();
+  if constexpr (MB > 0) return reinterpret_cast<const void*>(&msv_multi_kernel_mb<G, Q, MB>);
+  else return reinterpret_cast<const void*>(&msv_multi_kernel<G, Q>);
 }
 
 }  // namespace hmg
