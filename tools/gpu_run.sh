@@ -31,4 +31,9 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:vit_
 timeout 900 python tools/configs_bench.py 1,2,3,4,5 > $O/configs_$TAG.jsonl 2> $O/configs_$TAG.err
 timeout 300 python tools/fwd_bench.py > $O/fwd_bench_$TAG.jsonl 2>&1
 timeout 600 python tools/batch_bench.py 64 > $O/batch_bench_$TAG.jsonl 2>&1
+# summaries on the box (gpurun copies back at most 64 MiB): keep only the MSV report
+python tools/ncu_summary.py $O/*_$TAG.ncu-rep > $O/ncu_full_$TAG.md 2>&1
+python tools/launch_summary.py $O/launches_$TAG.csv "bench launch list ($TAG)" > $O/launches_$TAG.md 2>&1
+mkdir -p /tmp/ncu_reps_$TAG
+for f in $O/*_$TAG.ncu-rep; do case "$f" in *msv_fast_*) ;; *) mv "$f" /tmp/ncu_reps_$TAG/ ;; esac; done
 echo "done $TAG"
