@@ -292,7 +292,8 @@ struct MsvLong {
 
 // Minimum resident blocks per SM for a lane geometry: forcing 3 (<= 85 registers) lets a third
 // 256-thread block share the SM where the measured sweep gains (profiles/msv_minb_r01.jsonl:
-// G = 8, Q = 26: -7%; G = 16, Q = 16: -15%; G = 32, Q = 24 at 2 blocks: -6%); 0 = no bound.
+// G = 8, Q = 26: -7%; G = 16, Q = 16: -15%; G = 32, Q = 24 at 2 blocks: -6%; a fourth block at
+// G = 8, Q = 26 spills in the row loop: +31%); 0 = no bound.
 template <int G, int Q>
 constexpr int msv_min_blocks() {
   if (G == 4 && Q >= 8 && Q <= 10) return 3;
