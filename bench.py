@@ -15,6 +15,13 @@ length-balanced shard of an N x 550k DB (weak scaling).
 
 Prints ONE JSON line on rank 0.  --impl reference runs the CPU oracle (the
 reference arm of this tier) on a bounded sample of the same workload.
+
+The pipeline is captured once in a CUDA graph and replayed per timed step (--no-graph: eager).
+Beside the 8(a) headline the line carries (N = 1): `e2e` (hmg_pipeline_upload: the packed DB
+re-sent from pinned host memory, overlapped with the filter, plus the D2H of the results),
+`forward` (Fig 1 with the Forward stage, with its FP32 roofline), `batch` (the
+f4 many-profile leg), `cpu_baseline` (the oracle on the host cores) and `roofline` (the MSV
+kernel against the measured ALU-pipe peak, DRAM traffic from the committed ncu capture).
 """
 from __future__ import annotations
 

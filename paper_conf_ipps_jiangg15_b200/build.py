@@ -3,7 +3,8 @@
 Every .cu under csrc/ is compiled to an object (in parallel, one nvcc per file)
 with ``-gencode arch=compute_100a,code=sm_100a -lineinfo -O3`` and linked into
 ``paper_conf_ipps_jiangg15_b200/libhmg.so``.  No JIT cache is involved: the .so
-travels with the repo snapshot to the GPU box.
+travels with the repo snapshot to the GPU box.  ``HMG_NVCC_EXTRA`` appends nvcc flags (used by
+the tuning sweeps, e.g. ``-DMSV_MINB=...``; not needed for a normal build).
 """
 from __future__ import annotations
 
