@@ -1373,8 +1373,8 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2 * kUploadParts, &e);
     if (e) return cuda_status(e);
     if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2 * kUploadParts, st))) return cuda_status(e);
-    // overlapped upload: part boundaries (sorted indices) of about equal residues, part 0 >= the
-    // long lane; part k's words are one contiguous run of the image
+    // overlapped upload: part boundaries (sorted indices), part 0 >= the long lane; part k's
+    // words are one contiguous run of the image
     int64_t bnd[kUploadParts + 1] = {0};
     int nparts = 1;
     bnd[1] = n;
@@ -1382,11 +1382,15 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     cudaStream_t cs = nullptr;
     if (h_image) {
       nparts = std::max(2, std::min(kUploadParts, env_int("HMG_UPLOAD_PARTS", 6)));   // profiles/upload_parts_r01.jsonl
-      const int64_t per = (db->residues + nparts - 1) / nparts;
+      // a small first part (the filter waits for it; later parts land faster than MSV consumes
+      // them), then equal parts of the rest
+      const int first_pm = env_int("HMG_UPLOAD_FIRST_PERMILLE", 50);   // profiles/upload_parts_r01b.jsonl
+      const int64_t r0 = db->residues * first_pm / 1000;
+      const int64_t per = (db->residues - r0 + nparts - 2) / std::max(1, nparts - 1);
       int64_t acc = 0, k = 1;
       for (int64_t j = 0; j < n && k < nparts; ++j) {
         acc += db->len_sorted[j];
-        if (acc >= per * k && j + 1 >= nlong) bnd[k++] = j + 1;
+        if (acc >= r0 + per * (k - 1) && j + 1 >= nlong) bnd[k++] = j + 1;
       }
       while (k < nparts) bnd[k++] = n;
       bnd[nparts] = n;
