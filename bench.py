@@ -43,6 +43,7 @@ sys.path.insert(0, ROOT)
 METRIC = "MSV / P7Viterbi / pipeline GCUPS at 1/2/4/8 B200; fraction of int-SIMD roofline"
 ALU_LANES_PER_CLK_SM = 64        # measured: VIADDMNMX/VIMNMX3 issue at 64 lanes/clk/SM (profiles/intpeak)
 MSV_ALU_OPS_PER_CELL = 0.75      # VIADDMNMX.S16x2 (1 per 2 cells) + VIMNMX3.S16x2 (1 per 4 cells)
+VIT_ALU_OPS_PER_CELL = 4.25      # s16x2 pair kernel: M 4, I 2, D 2, R 1/2 per cell pair
 FP32_LANES_PER_CLK_SM = 128      # B200 FP32 FMA lanes per SM per clock (4 SMSPs x 32)
 FWD_FLOPS_PER_CELL = 16          # Forward recurrence: M 4 mul + 3 add + 1 mul, I 2 mul + 1 add,
                                  # D 2 mul + 1 add, E 2 add
@@ -520,6 +521,10 @@ def main():
                        "msv_redo_ms": round(st["msv_redo"], 4),
                        "flags_compaction_ms": round(st["msv_flags_compaction"], 4),
                        "vit_kernel_ms": round(vit_ms, 4), "vit_gcups": round(vit_gcups, 2) if vit_gcups else None,
+                       "vit_roofline_frac": (round(vit_gcups * 1e9 * VIT_ALU_OPS_PER_CELL / (p_int * 1e12), 4)
+                                             if vit_gcups else None),
+                       "vit_roofline_note": "vs the ALU-pipe peak at %.2f ops/cell (s16x2 pair kernel); the "
+                                            "survivor stage is schedule-bound (DESIGN.md 4.3)" % VIT_ALU_OPS_PER_CELL,
                        "vit_flags_ms": round(st["vit_flags"], 4),
                        "vit_pair_kernel": P.quant()["vit_pair_lanes"] > 0, "vit_s32_rescored": int(redo),
                        "survivors": int(ns_all), "survivor_frac": round(ns_all / max(n_all, 1), 5),
