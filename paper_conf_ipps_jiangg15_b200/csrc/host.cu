@@ -174,6 +174,24 @@ int env_int(const char* name, int dflt) {
   return v ? atoi(v) : dflt;
 }
 
+// Stream-ordered scratch (Scratch below) comes from the device's default memory pool; its default
+// release threshold (0) returns the memory to the driver at every synchronisation, so each eager
+// call would map its scratch again (milliseconds for the DB-sized buffers).  Keep it cached.
+void keep_pool_cached(int device) {
+  static std::mutex mu;
+  static std::vector<bool> done;
+  std::lock_guard<std::mutex> g(mu);
+  if ((int)done.size() <= device) done.resize(device + 1, false);
+  if (done[device]) return;
+  cudaMemPool_t pool = nullptr;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  cudaGetLastError();
+  done[device] = true;
+}
+
 // ---------------------------------------------------------------- kernel geometry
 void msv_geometry(int M, int* G, int* Q) {
   // lane-group size from the G sweep on the config-2 DB (profiles/msv_sweep_r01.txt)
@@ -735,6 +753,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
       return ndev == 0 ? HMG_EUNSUPPORTED : HMG_EINVAL;
     }
   }
+  if (device >= 0) keep_pool_cached(device);
   hmg_profile* p = new (std::nothrow) hmg_profile();
   if (!p) return HMG_ENOMEM;
   p->M = M;
@@ -1116,6 +1135,7 @@ hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, i
   }
   for (int64_t i = 0; i < (nseq ? off[nseq] - off[0] : 0); ++i)
     if (dsq[off[0] + i] > 28) return HMG_EINVAL;
+  if (device >= 0) keep_pool_cached(device);
   hmg_db* db = new (std::nothrow) hmg_db();
   if (!db) return HMG_ENOMEM;
   db->device = device;
