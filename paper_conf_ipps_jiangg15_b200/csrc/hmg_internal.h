@@ -237,7 +237,7 @@ cudaError_t select_redo_pairs(const uint8_t* raw_sorted, int64_t n, int64_t* lis
                               cudaStream_t st);
 cudaError_t msv_flags_multi(const uint8_t* raw_sorted, int nprof, const int32_t* len, const int32_t* order,
                             int64_t nseq, const uint16_t* const* thr, const int* rowmap, uint8_t* raw_out,
-                            uint8_t* pass_out, cudaStream_t st);
+                            uint8_t* pass_out, cudaStream_t st, uint8_t* pass_sorted = nullptr);
 
 // pipeline helpers (pipeline.cu)
 cudaError_t select_redo(const uint8_t* raw_sorted, int64_t n, int32_t* list, int64_t* count, void* tmp,
@@ -250,6 +250,9 @@ cudaError_t vit_finish(const int16_t* raw_sorted, const int32_t* list, const int
                        uint8_t* pass_out, uint8_t* flags_out, cudaStream_t st, uint8_t* pass_sorted = nullptr);
 cudaError_t compact_flags(const uint8_t* flag_sorted, int64_t n, const int32_t* order, int32_t* ids_sorted,
                           int32_t* ids_caller, int64_t* count, void* tmp, cudaStream_t st);
+size_t compact_rows_tmp_bytes(int64_t n, int rows);
+cudaError_t compact_rows(const uint8_t* flag, int rows, int64_t n, const int32_t* order, int32_t* ids_sorted,
+                         int32_t* ids_caller, int64_t* counts, const int* rowmap, void* tmp, cudaStream_t st);
 
 // Forward stage (forward.cu)
 // T = threads per sequence (8: sub-warp lane groups; 32 W: W warps)

@@ -1855,8 +1855,19 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
                           st);
       mark(3, st);
     } else {
-      // per profile (Fig 1): pass flags + stable survivor compaction of its row, Viterbi filter on the
-      // survivors, flags; the profiles' chains run concurrently on the side streams
+      // Fig 1 per profile: pass flags of every row and the stable survivor compaction of every row
+      // in four launches on st, then each profile's Viterbi filter on its survivors; the profiles'
+      // Viterbi chains run concurrently on the side streams
+      auto* fs = (uint8_t*)S.get((size_t)nprof * (size_t)n, &e);
+      auto* surv_all = (int32_t*)S.get(sizeof(int32_t) * (size_t)nprof * (size_t)n, &e);
+      void* ctmp = S.get(compact_rows_tmp_bytes(n, nprof), &e);
+      if (e) return cuda_status(e);
+      if ((e = msv_flags_multi(raw_sorted, nprof, db->d_len, db->d_order, n, d_thr, d_rows, raw, tail->flags, st,
+                               fs)))
+        return cuda_status(e);
+      if ((e = compact_rows(fs, nprof, n, db->d_order, surv_all, tail->survivor_ids, tail->n_survivors, d_rows, ctmp,
+                            st)))
+        return cuda_status(e);
       std::vector<const int32_t*> tv(nprof);
       for (int r = 0; r < nprof; ++r) {
         hmg_status s = vit_thr_table(const_cast<hmg_profile*>(profs[rows[r]]), db, tail->F2, &tv[r]);
@@ -1876,14 +1887,13 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
       }
       {
         std::vector<Scratch*> SS;
-        struct Bufs { int32_t* surv; int16_t* vraw; void* tmp; uint8_t* vpass; int32_t* fl; };
+        struct Bufs { int16_t* vraw; void* tmp; uint8_t* vpass; int32_t* fl; };
         std::vector<Bufs> B;
         hmg_status s = HMG_OK;
         for (int k = 0; k < std::max(ns, 1); ++k) {
           cudaStream_t sk = ns > 1 ? side[k] : st;
           SS.push_back(new Scratch(sk));
           Bufs b{};
-          b.surv = (int32_t*)SS.back()->get(sizeof(int32_t) * (size_t)n, &e);
           b.vraw = (int16_t*)SS.back()->get(sizeof(int16_t) * (size_t)n, &e);
           b.tmp = SS.back()->get(scan_tmp_bytes(n) + (size_t)n + 16, &e);
           if (tail->fwd_nats) {
@@ -1898,13 +1908,11 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
           const int i = rows[r];
           const hmg_profile* pi = profs[i];
           const size_t ro = (size_t)i * n;
-          e = msv_finish(raw_sorted + (size_t)r * n, db->d_len, db->d_order, n, thr[r], raw + ro, tail->flags + ro,
-                         B[k].surv, tail->n_survivors + i, tail->survivor_ids + ro, B[k].tmp, sk);
-          if (e) break;
-          s = run_vit(pi, db, B[k].surv, tail->n_survivors + i, sk, B[k].vraw, *SS[k], nullptr, 0, false, n);
+          const int32_t* surv = surv_all + (size_t)r * n;
+          s = run_vit(pi, db, surv, tail->n_survivors + i, sk, B[k].vraw, *SS[k], nullptr, 0, false, n);
           if (s != HMG_OK) break;
           if (tail->fwd_nats && (e = cudaMemsetAsync(B[k].vpass, 0, (size_t)n, sk))) break;
-          e = vit_finish(B[k].vraw, B[k].surv, tail->n_survivors + i, n, db->d_len, db->d_order, tv[r],
+          e = vit_finish(B[k].vraw, surv, tail->n_survivors + i, n, db->d_len, db->d_order, tv[r],
                          tail->vit_raw + ro, nullptr, tail->flags + ro, sk, tail->fwd_nats ? B[k].vpass : nullptr);
           if (e || !tail->fwd_nats) continue;
           // Forward stage on this profile's Viterbi passes (Fig 1)

@@ -140,7 +140,8 @@ cudaError_t select_redo_pairs(const uint8_t* raw_sorted, int64_t n, int64_t* lis
 __global__ void msv_flags_multi_kernel(const uint8_t* __restrict__ raw, int nprof, const int32_t* __restrict__ len,
                                        const int32_t* __restrict__ order, int64_t nseq,
                                        const uint16_t* const* __restrict__ thr, const int* __restrict__ rowmap,
-                                       uint8_t* __restrict__ raw_out, uint8_t* __restrict__ pass_out) {
+                                       uint8_t* __restrict__ raw_out, uint8_t* __restrict__ pass_out,
+                                       uint8_t* __restrict__ pass_sorted) {
   const int p = blockIdx.y;                    // row of raw (bucket order) -> caller profile rowmap[p]
   const uint8_t* r = raw + (size_t)p * nseq;
   const uint16_t* th = thr ? thr[p] : nullptr;
@@ -149,20 +150,23 @@ __global__ void msv_flags_multi_kernel(const uint8_t* __restrict__ raw, int npro
     const int v = r[k];
     const size_t c = ro + order[k];
     raw_out[c] = (uint8_t)v;
-    if (pass_out) pass_out[c] = th ? (uint8_t)(v == 255 || v >= (int)th[len[k]]) : 0;
+    const uint8_t pv = th ? (uint8_t)(v == 255 || v >= (int)th[len[k]]) : 0;
+    if (pass_out) pass_out[c] = pv;
+    if (pass_sorted) pass_sorted[(size_t)p * nseq + k] = pv;   // row p (bucket order), sorted order
   }
 }
 
 cudaError_t msv_flags_multi(const uint8_t* raw_sorted, int nprof, const int32_t* len, const int32_t* order,
                             int64_t nseq, const uint16_t* const* thr, const int* rowmap, uint8_t* raw_out,
-                            uint8_t* pass_out, cudaStream_t st) {
+                            uint8_t* pass_out, cudaStream_t st, uint8_t* pass_sorted) {
   if (nseq <= 0 || nprof <= 0) return cudaSuccess;
   int64_t bx = (nseq + 255) / 256;
   const int64_t cap = std::max<int64_t>(1, 4096 / nprof);
   if (bx > cap) bx = cap;
   g_launches += 1;
   msv_flags_multi_kernel<<<dim3((unsigned)bx, (unsigned)nprof), 256, 0, st>>>(raw_sorted, nprof, len, order, nseq,
-                                                                             thr, rowmap, raw_out, pass_out);
+                                                                             thr, rowmap, raw_out, pass_out,
+                                                                             pass_sorted);
   return cudaGetLastError();
 }
 

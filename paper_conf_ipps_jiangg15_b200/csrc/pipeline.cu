@@ -22,7 +22,12 @@ size_t scan_tmp_bytes(int64_t n) {
   return (size_t)(2 * nt + 2) * sizeof(int64_t);
 }
 
-__global__ void count_kernel(const uint8_t* __restrict__ flag, int64_t n, int64_t* __restrict__ tilecnt) {
+// Row y = blockIdx.y of a [rows][n] flag matrix (one row for the single-profile calls): flags at
+// y * n, tile counts / offsets at y * tstride, outputs of caller row rowmap[y] (rowmap NULL: y).
+__global__ void count_kernel(const uint8_t* __restrict__ flag, int64_t n, int64_t* __restrict__ tilecnt,
+                             int64_t tstride) {
+  flag += (size_t)blockIdx.y * n;
+  tilecnt += (size_t)blockIdx.y * tstride;
   const int64_t t0 = (int64_t)blockIdx.x * kTile;
   int c = 0;
   for (int i = threadIdx.x; i < kTile; i += kThreads) {
@@ -42,7 +47,10 @@ __global__ void count_kernel(const uint8_t* __restrict__ flag, int64_t n, int64_
 
 // exclusive scan of tile counts by one block; writes total to *count
 __global__ void scan_kernel(const int64_t* __restrict__ tilecnt, int64_t ntiles, int64_t* __restrict__ tileoff,
-                            int64_t* __restrict__ count) {
+                            int64_t* __restrict__ count, int64_t tstride, const int* __restrict__ rowmap) {
+  tilecnt += (size_t)blockIdx.x * tstride;
+  tileoff += (size_t)blockIdx.x * tstride;
+  count += rowmap ? rowmap[blockIdx.x] : (int)blockIdx.x;
   __shared__ int64_t carry;
   __shared__ int64_t wsum[kThreads / 32];
   if (threadIdx.x == 0) carry = 0;
@@ -72,7 +80,11 @@ __global__ void scan_kernel(const int64_t* __restrict__ tilecnt, int64_t ntiles,
 // stable scatter: ids_sorted[j] = k, ids_caller[j] = order[k] for the j-th flagged k
 __global__ void scatter_kernel(const uint8_t* __restrict__ flag, int64_t n, const int64_t* __restrict__ tileoff,
                                const int32_t* __restrict__ order, int32_t* __restrict__ ids_sorted,
-                               int32_t* __restrict__ ids_caller) {
+                               int32_t* __restrict__ ids_caller, int64_t tstride, const int* __restrict__ rowmap) {
+  flag += (size_t)blockIdx.y * n;
+  tileoff += (size_t)blockIdx.y * tstride;
+  if (ids_sorted) ids_sorted += (size_t)blockIdx.y * n;
+  if (ids_caller) ids_caller += (size_t)(rowmap ? rowmap[blockIdx.y] : (int)blockIdx.y) * n;
   const int64_t t0 = (int64_t)blockIdx.x * kTile;
   __shared__ int64_t base;
   __shared__ int wsum[kThreads / 32];
@@ -108,11 +120,36 @@ static cudaError_t compact(const uint8_t* flag, int64_t n, const int32_t* order,
   int64_t* tileoff = tilecnt + nt + 1;
   if (nt == 0) return cudaMemsetAsync(count, 0, sizeof(int64_t), st);
   g_launches += 1;
-  count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(flag, n, tilecnt);
+  count_kernel<<<(unsigned)nt, kThreads, 0, st>>>(flag, n, tilecnt, 0);
   g_launches += 1;
-  scan_kernel<<<1, kThreads, 0, st>>>(tilecnt, nt, tileoff, count);
+  scan_kernel<<<1, kThreads, 0, st>>>(tilecnt, nt, tileoff, count, 0, nullptr);
   g_launches += 1;
-  scatter_kernel<<<(unsigned)nt, kThreads, 0, st>>>(flag, n, tileoff, order, ids_sorted, ids_caller);
+  scatter_kernel<<<(unsigned)nt, kThreads, 0, st>>>(flag, n, tileoff, order, ids_sorted, ids_caller, 0, nullptr);
+  return cudaGetLastError();
+}
+
+size_t compact_rows_tmp_bytes(int64_t n, int rows) {
+  const int64_t nt = (n + kTile - 1) / kTile;
+  return (size_t)rows * 2 * (size_t)(nt + 1) * sizeof(int64_t) + 16;
+}
+
+// Stable compaction of every row of a [rows][n] sorted-order flag matrix in three launches
+// (many-profile pipeline): ids_sorted [rows][n] (row y), ids_caller / counts at caller row rowmap[y].
+cudaError_t compact_rows(const uint8_t* flag, int rows, int64_t n, const int32_t* order, int32_t* ids_sorted,
+                         int32_t* ids_caller, int64_t* counts, const int* rowmap, void* tmp, cudaStream_t st) {
+  const int64_t nt = (n + kTile - 1) / kTile;
+  if (rows <= 0) return cudaSuccess;
+  const int64_t ts = nt + 1;
+  int64_t* tilecnt = reinterpret_cast<int64_t*>(tmp);
+  int64_t* tileoff = tilecnt + (size_t)rows * ts;
+  if (nt == 0) return cudaSuccess;
+  g_launches += 1;
+  count_kernel<<<dim3((unsigned)nt, (unsigned)rows), kThreads, 0, st>>>(flag, n, tilecnt, ts);
+  g_launches += 1;
+  scan_kernel<<<(unsigned)rows, kThreads, 0, st>>>(tilecnt, nt, tileoff, counts, ts, rowmap);
+  g_launches += 1;
+  scatter_kernel<<<dim3((unsigned)nt, (unsigned)rows), kThreads, 0, st>>>(flag, n, tileoff, order, ids_sorted,
+                                                                          ids_caller, ts, rowmap);
   return cudaGetLastError();
 }
 
