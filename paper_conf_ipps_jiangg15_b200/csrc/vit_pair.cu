@@ -1,6 +1,9 @@
 // vit_pair.cu -- launcher of the s16x2 pair Viterbi kernel (vit_pair.cuh).
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cstdlib>
+
 #include "vit_pair.cuh"
 
 namespace hmg {
@@ -35,6 +38,8 @@ cudaError_t launch_vit_pair(int G, int Q, bool scan, const VitArgs& a, cudaStrea
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, 128, smem);
   if (e != cudaSuccess) return e;
   if (per < 1) per = 1;
+  // (fewer blocks per SM -- faster rows for the longest survivors, less throughput -- measured
+  //  slower at 1 / 2 / 3 blocks: profiles/vit_bps_r01.jsonl)
   const int64_t grid = (int64_t)nsm * per;
   void* args[] = {const_cast<VitArgs*>(&a)};
   g_launches += 1;
