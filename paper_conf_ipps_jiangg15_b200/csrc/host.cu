@@ -1356,7 +1356,7 @@ static cudaStream_t* side_streams(int device);
 // h_image (optional): pinned host copy of the packed DB image (hmg_db_image); it is uploaded in
 // kUploadParts length-ordered parts on a side stream while the MSV kernel scores the parts that
 // have landed (one launch per part), so the H2D overlaps the filter.
-constexpr int kUploadParts = 8;     // capacity; parts used: HMG_UPLOAD_PARTS (default 6)
+constexpr int kUploadParts = 12;    // capacity; parts used: HMG_UPLOAD_PARTS (default 6)
 
 static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
                                 uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
@@ -1405,12 +1405,19 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       // a small first part (the filter waits for it; later parts land faster than MSV consumes
       // them), then equal parts of the rest
       const int first_pm = env_int("HMG_UPLOAD_FIRST_PERMILLE", 50);   // profiles/upload_parts_r01b.jsonl
+      // the rest in parts whose sizes follow a geometric ratio HMG_UPLOAD_GROW / 1000 (1000 = equal
+      // parts); a ratio below 1 shrinks the last parts, whose MSV cannot start before they land
       const int64_t r0 = db->residues * first_pm / 1000;
-      const int64_t per = (db->residues - r0 + nparts - 2) / std::max(1, nparts - 1);
+      const double g = std::max(1, env_int("HMG_UPLOAD_GROW", 1000)) / 1000.0;
+      double cut[kUploadParts] = {0.0}, wsum = 0.0, wk = 1.0;
+      for (int q = 1; q < nparts; ++q, wk *= g) wsum += wk;
+      wk = 1.0;
+      for (int q = 1; q < nparts; ++q, wk *= g)
+        cut[q] = (q > 1 ? cut[q - 1] : (double)r0) + (double)(db->residues - r0) * wk / wsum;
       int64_t acc = 0, k = 1;
       for (int64_t j = 0; j < n && k < nparts; ++j) {
         acc += db->len_sorted[j];
-        if (acc >= r0 + per * (k - 1) && j + 1 >= nlong) bnd[k++] = j + 1;
+        if ((k == 1 ? acc >= r0 : (double)acc >= cut[k - 1]) && j + 1 >= nlong) bnd[k++] = j + 1;
       }
       while (k < nparts) bnd[k++] = n;
       bnd[nparts] = n;
