@@ -258,10 +258,14 @@ hmg_status hmg_stage_times(double* ms);
 hmg_status hmg_stage_counts(int64_t* counts);
 
 /* hmg_db_upload + hmg_pipeline with the upload overlapped: the packed image (host, pinned; from
- * hmg_db_image of this DB) is copied in 6 length-ordered parts of about equal residues on a side
- * stream, and the MSV kernel scores each part as soon as it has landed (the long lane with the
- * first part), so the H2D of parts 2-6 hides behind the filter.  Outputs and results are
- * hmg_pipeline's.  The image must stay valid until the call's work on `stream` has completed. */
+ * hmg_db_image of this DB) is copied in length-ordered parts on a side stream (a first part of
+ * 5% of the residues, then 5 parts of about equal residues; env HMG_UPLOAD_PARTS / _FIRST_PERMILLE
+ * / _GROW), each followed by a 4-byte copy that sets its landing flag; ONE MSV launch scores every
+ * part, each batch of sequences waiting on its part's flag (the long lane starts with the first
+ * part), so the H2D of the later parts hides behind the filter with no kernel boundary per part
+ * (HMG_UPLOAD_GATED=0: one MSV launch per part).
+ * Outputs and results are hmg_pipeline's.  The image must stay valid until the call's work on
+ * `stream` has completed. */
 hmg_status hmg_pipeline_upload(const hmg_profile* p, hmg_db* db, const uint32_t* image, double F1, double F2,
                                void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
                                int32_t* survivor_ids, int64_t* n_survivors);

@@ -21,6 +21,8 @@ constexpr int16_t kNegE = -16384;   // "minus infinity" emission / carry of the 
 constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
 
 // ---------------------------------------------------------------- MSV kernel arguments
+constexpr int kMaxGates = 12;   // = kUploadParts (host.cu)
+
 struct MsvArgs {
   const uint32_t* words;     // packed residues
   const uint32_t* woff16;    // [nseq] sorted: word offset / 4 (16-byte units)
@@ -37,6 +39,11 @@ struct MsvArgs {
   const int32_t* list;       // exact kernel: sorted indices to redo
   const int64_t* nlist;      // exact kernel: device count
   uint8_t* scratch;          // exact kernel: per-warp row buffers
+  // fast kernel, overlapped upload (hmg_pipeline_upload): the sorted range is in ngate parts,
+  // part q = [.., gate_end[q]); a batch waits until gate_flag[q] != 0 (set behind part q's H2D)
+  int ngate;
+  const unsigned* gate_flag;
+  long long gate_end[kMaxGates];
 };
 
 // Many-profile MSV (msv_multi.cuh): a bucket of profiles with one lane geometry

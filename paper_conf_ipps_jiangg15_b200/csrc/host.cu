@@ -459,11 +459,15 @@ double mean_len(const hmg_db* db) { return db->nseq ? (double)db->residues / (do
 // first pipe_nlong sequences are scored by the pipeline long lane instead.
 hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S,
                         int64_t pipe_nlong, bool pdl = false, bool mark0 = true,
-                        unsigned long long* ctr_zeroed = nullptr, int64_t end = -1) {
+                        unsigned long long* ctr_zeroed = nullptr, int64_t end = -1,
+                        int ngate = 0, const unsigned* gate_flag = nullptr, const int64_t* gate_end = nullptr) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
   a.raw = raw_sorted;
+  a.ngate = ngate;
+  a.gate_flag = gate_flag;
+  for (int q = 0; q < ngate && q < kMaxGates; ++q) a.gate_end[q] = gate_end[q];
   if (end >= 0) a.nseq = end;          // sorted range [pipe_nlong, end) only (overlapped upload)
   if (pipe_nlong >= 0) {
     a.nlong = pipe_nlong;
@@ -1353,10 +1357,27 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
 
 static cudaStream_t* side_streams(int device);
 
+// The overlapped upload marks each part as landed by a 4-byte H2D copy of the value 1 into a
+// device flag, queued on the copy stream right behind the part (the copy engine completes copies
+// of a stream in order), which the single gated MSV launch polls.  Source: one pinned word.
+static const unsigned* pinned_one() {
+  static unsigned* one = [] {
+    unsigned* h = nullptr;
+    if (cudaHostAlloc(&h, sizeof(unsigned), cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      return (unsigned*)nullptr;
+    }
+    *h = 1u;
+    return h;
+  }();
+  return one;
+}
+
 // h_image (optional): pinned host copy of the packed DB image (hmg_db_image); it is uploaded in
 // kUploadParts length-ordered parts on a side stream while the MSV kernel scores the parts that
 // have landed (one launch per part), so the H2D overlaps the filter.
 constexpr int kUploadParts = 12;    // capacity; parts used: HMG_UPLOAD_PARTS (default 6)
+static_assert(kUploadParts <= kMaxGates, "one landing gate per upload part");
 
 static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
                                 uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
@@ -1390,9 +1411,12 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
                            (p->long_pair || (!p->vit_generic && p->vit_W == 0)) &&
                            !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
-    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2 * kUploadParts, &e);
+    // part counters (2 per part) + the gated launch's landing flags (u32, one per part)
+    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 3 * kUploadParts, &e);
     if (e) return cuda_status(e);
-    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2 * kUploadParts, st))) return cuda_status(e);
+    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 3 * kUploadParts, st))) return cuda_status(e);
+    unsigned* gate_flag = reinterpret_cast<unsigned*>(mctr + 2 * kUploadParts);
+    const unsigned* one = h_image && env_int("HMG_UPLOAD_GATED", 0) ? pinned_one() : nullptr;
     // overlapped upload: part boundaries (sorted indices), part 0 >= the long lane; part k's
     // words are one contiguous run of the image
     int64_t bnd[kUploadParts + 1] = {0};
@@ -1436,6 +1460,8 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
         if (w1 > w0 && (e = cudaMemcpyAsync(db->d_words + w0, h_image + w0, (size_t)(w1 - w0) * 4,
                                             cudaMemcpyHostToDevice, cs)))
           return cuda_status(e);
+        if (one && (e = cudaMemcpyAsync(gate_flag + q, one, sizeof(unsigned), cudaMemcpyHostToDevice, cs)))
+          return cuda_status(e);                    // landing flag of part q, behind its data
         if ((e = cudaEventRecord(up_ev[q], cs))) return cuda_status(e);
       }
       if ((e = cudaStreamWaitEvent(st, up_ev[0], 0))) return cuda_status(e);
@@ -1485,7 +1511,17 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV
       if (s != HMG_OK) return s;
     } else {
-      for (int q = 0; q < nparts; ++q) {          // MSV of each part once it has landed
+      if (one) {       // one launch over every part: each batch waits on its part's landing flag
+        int64_t gend[kUploadParts];
+        for (int q = 0; q < nparts; ++q) gend[q] = bnd[q + 1];
+        if (nlong < n) {
+          s = run_msv_fast(p, db, ms, raw_sorted, S, nlong, false, false, mctr, n, nparts, gate_flag, gend);
+          if (s != HMG_OK) return s;
+        }
+        // join the copy stream (after the launch, which must not wait for the upload)
+        if ((e = cudaStreamWaitEvent(ms, up_ev[nparts - 1], 0))) return cuda_status(e);
+      }
+      for (int q = 0; q < nparts && !one; ++q) {  // else: MSV of each part once it has landed
         if ((e = cudaStreamWaitEvent(ms, up_ev[q], 0))) return cuda_status(e);
         const int64_t lo = std::max(bnd[q], nlong), hi = bnd[q + 1];
         if (hi > lo) {

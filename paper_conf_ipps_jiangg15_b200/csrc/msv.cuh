@@ -76,6 +76,8 @@ __device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z
 // Residue stream of one sequence: 16-byte quads of packed words (24 residues) fetched two
 // quads ahead, so the DRAM/L2 latency of the residue stream hides behind >= 24 DP rows even
 // for short models.  Words past the sequence are all-31 (pad rows).
+// (L2-only loads, not the read-only path: under hmg_pipeline_upload the image lands while the MSV
+//  kernel runs, and a line shared with an earlier part may already sit in L1)
 struct ResStream {
   const uint4* p;
   int nq;
@@ -84,16 +86,26 @@ struct ResStream {
   __device__ __forceinline__ void init(const uint32_t* wp, int nw) {
     p = reinterpret_cast<const uint4*>(wp);
     nq = (nw + 3) / 4;
-    cur = nq > 0 ? __ldg(p) : pad();
-    nxt = nq > 1 ? __ldg(p + 1) : pad();
+    cur = nq > 0 ? __ldcg(p) : pad();
+    nxt = nq > 1 ? __ldcg(p + 1) : pad();
   }
   __device__ __forceinline__ uint4 next(int iq) {   // quad iq, prefetching iq + 2
     const uint4 r = cur;
     cur = nxt;
-    nxt = (iq + 2 < nq) ? __ldg(p + iq + 2) : pad();
+    nxt = (iq + 2 < nq) ? __ldcg(p + iq + 2) : pad();
     return r;
   }
 };
+
+// spin (bounded: ~2 s, never a hang) until a flag written by a stream memory operation is set
+__device__ __forceinline__ void gate_wait(const unsigned* f) {
+  for (int it = 0;; ++it) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+    if (v != 0u || it > (1 << 22)) break;
+    __nanosleep(500);
+  }
+}
 
 __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
@@ -333,6 +345,13 @@ __device__ __forceinline__ void msv_fast_body(const MsvArgs& a) {
     if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);
     b = __shfl_sync(0xffffffffu, b, 0);
     if (first + (long long)b >= a.nseq) break;
+    if (a.ngate > 0) {                 // overlapped upload: wait until this batch's part has landed
+      const long long last = min(first + (long long)b + NG, (long long)a.nseq) - 1;
+      int q = 0;
+      while (q < a.ngate - 1 && last >= a.gate_end[q]) ++q;
+      if (lane == 0) gate_wait(a.gate_flag + q);
+      __syncwarp();
+    }
     msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
   }
 }

@@ -575,15 +575,18 @@ def test_vit_pair_maxplus_scan(M, monkeypatch):
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
 
 
-@pytest.mark.parametrize("cfg,sched", [(1, None), (3, None), (3, (12, 700)), (3, (2, 1500))])
+@pytest.mark.parametrize("cfg,sched", [(1, None), (3, None), (3, (12, 700, 1)), (3, (2, 1500, 1)),
+                                       (3, (6, 1000, 0)), (1, (12, 1000, 0))])
 def test_pipeline_upload_overlapped_equals_pipeline(cfg, sched, monkeypatch):
     """hmg_pipeline_upload (packed image re-sent from pinned host memory in length-ordered parts,
     MSV per part as it lands, long lane alongside) gives hmg_pipeline's outputs exactly; the device
     image is scrubbed first so every residue read must come from this call's upload.  `sched`
-    overrides the part schedule (HMG_UPLOAD_PARTS, HMG_UPLOAD_GROW: shrinking / growing parts)."""
+    overrides the part schedule (HMG_UPLOAD_PARTS, HMG_UPLOAD_GROW: shrinking / growing parts;
+    HMG_UPLOAD_GATED: one MSV launch waiting on per-part landing flags, or one launch per part)."""
     if sched is not None:
         monkeypatch.setenv("HMG_UPLOAD_PARTS", str(sched[0]))
         monkeypatch.setenv("HMG_UPLOAD_GROW", str(sched[1]))
+        monkeypatch.setenv("HMG_UPLOAD_GATED", str(sched[2]))
     prof, db = synth.config(cfg)
     dsq, off = db.materialize()
     ev = _calibrate(prof) if cfg == 1 else (-9.5, math.log(2), -9.0, math.log(2))
