@@ -123,7 +123,7 @@ __global__ void __launch_bounds__((W == 1 ? GL : 32 * W) * S, 1) fwd_kernel(cons
     };
     const int nw = (L + 5) / 6, nww = (Lw + 5) / 6;
     for (int w0 = 0; w0 < nww; w0 += GL) {
-      const uint32_t wreg = (w0 + lane < nw) ? __ldg(wp + w0 + lane) : 0u;
+      const uint32_t wreg = (w0 + lane < nw) ? __ldcg(wp + w0 + lane) : 0u;
       const int wend = min(GL, nww - w0);
 #pragma unroll 1
       for (int j = 0; j < wend; ++j) {

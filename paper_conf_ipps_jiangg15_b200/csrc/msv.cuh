@@ -266,7 +266,7 @@ __device__ __forceinline__ bool msv_chunk(const MsvArgs& a, const uint32_t* __re
   const int wb = max(0, r0 - warm) / 6;        // first warm-up word
   const int we = min(nw, (r1 + 5) / 6);
   for (int blk = wb; blk < we; ++blk) {
-    const uint32_t w = __ldg(wp + blk);
+    const uint32_t w = __ldcg(wp + blk);
     const bool counting = blk >= wc;
 #pragma unroll
     for (int j = 0; j < 6; ++j) {

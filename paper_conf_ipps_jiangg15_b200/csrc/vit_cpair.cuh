@@ -183,10 +183,10 @@ __global__ void __launch_bounds__(32 * W * SG, 1) vit_cpair_kernel(const VitArgs
     uint32_t nbM = 0u, nbI = 0u, nbD = 0u;                        // lane 0: diagonal carries
     int par = 0;
     const int nw = (L + 5) / 6;
-    uint32_t wnxt = __ldg(wp);
+    uint32_t wnxt = __ldcg(wp);
     for (int iw = 0; iw < nw && state == 0; ++iw) {
      uint32_t wv = wnxt;
-     wnxt = iw + 1 < nw ? __ldg(wp + iw + 1) : ~0u;
+     wnxt = iw + 1 < nw ? __ldcg(wp + iw + 1) : ~0u;
 #pragma unroll 1
      for (int j = 0; j < 6; ++j) {
       const int x = wv & 31;                       // block-uniform: uniform branches below

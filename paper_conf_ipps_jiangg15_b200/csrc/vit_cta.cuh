@@ -132,13 +132,13 @@ __global__ void __launch_bounds__(32 * W, (W <= 8 ? 2 : 1)) vit_cta_kernel(const
     // row -1 (all -inf) as seen from the right-hand warp
     int nbM = kNegW, nbI = kNegW, nbD = kNegW;
     int par = 0;
-    uint32_t wcur = __ldg(wp), wnxt = L > 6 ? __ldg(wp + 1) : ~0u;
+    uint32_t wcur = __ldcg(wp), wnxt = L > 6 ? __ldcg(wp + 1) : ~0u;
     for (int i = 0; i < L; ++i) {
       const int j6 = i % 6;
       const int x = (wcur >> (5 * j6)) & 31;
       if (j6 == 5) {                              // next word; prefetch the one after it
         wcur = wnxt;
-        wnxt = (i / 6 + 2) * 6 < L ? __ldg(wp + i / 6 + 2) : ~0u;
+        wnxt = (i / 6 + 2) * 6 < L ? __ldcg(wp + i / 6 + 2) : ~0u;
       }
       const uint32_t* rowp = x < 20 ? tab + x * S::ROWW
                                     : (x == 26 ? tab + 20 * S::ROWW
