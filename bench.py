@@ -540,7 +540,7 @@ def main():
                        "vit_roofline_frac": (round(vit_gcups * 1e9 * VIT_ALU_OPS_PER_CELL / (p_int * 1e12), 4)
                                              if vit_gcups else None),
                        "vit_roofline_note": "vs the ALU-pipe peak at %.2f ops/cell (s16x2 pair kernel); the "
-                                            "survivor stage is schedule-bound (DESIGN.md 4.3)" % VIT_ALU_OPS_PER_CELL,
+                                            "survivor stage also carries the tail of its longest rows (DESIGN.md 4.3)" % VIT_ALU_OPS_PER_CELL,
                        "vit_flags_ms": round(st["vit_flags"], 4),
                        "vit_pair_kernel": P.quant()["vit_pair_lanes"] > 0, "vit_s32_rescored": int(redo),
                        "survivors": int(ns_all), "survivor_frac": round(ns_all / max(n_all, 1), 5),
