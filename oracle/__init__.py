@@ -10,12 +10,16 @@ marshals numpy arrays through ctypes.
 
 Every function cites the paper passage it follows (P:NNN = PAPER.md line).
 Parity status per function:
-  quantisation constants ........ pinned (closed forms, tests/test_oracle_quant.py)
-  MSV DP ......................... pinned (brute-force path enumeration, wide-int
-                                   recompute, invariants, closed form at L=1)
+  quantisation constants ........ pinned (closed forms, tests/test_oracle.py)
+  MSV DP ......................... pinned (brute-force path enumeration incl. segments
+                                   chained through J above base 190, wide-int recompute,
+                                   invariants, closed forms at L=1 and for two segments)
   Viterbi DP ..................... pinned (brute-force Plan-7 paths, wide-int
                                    recompute, ungapped special case)
-  nats / null1 / Gumbel / pass ... pinned (closed forms, textbook Gumbel)
+  nats / null1 / Gumbel / pass ... pinned (closed forms, golden VF-nats table written by
+                                   tests/golden/make_vit_nats.py, textbook Gumbel, direct
+                                   MSV / Viterbi pass decisions over a (raw, L, mu, F) grid,
+                                   statistical pass fractions at F1 and F2)
   Forward score (f2) ............. pinned (brute-force sum over all Plan-7 paths with
                                    N/J/C loops, closed form for a one-node model)
   agreement with HMMER 3.0 itself  parity unpinned (no HMMER source or scores

@@ -37,14 +37,16 @@ def s16(v):
 
 
 # ----------------------------------------------------------------------------- MSV
-def msv_brute(cost, bias, tbm, tec, tjb, dsq):
+def msv_brute(cost, bias, tbm, tec, tjb, dsq, reenter=True):
     """Max over ordered lists of row-disjoint ungapped diagonal segments.
 
     A segment enters at row i, node k from B (value 190 - tjb from N, or
     J - tjb from the previous segment's J value), loses tbm (B->M_k), and
     walks the diagonal (i, k), (i+1, k+1), ...; each cell adds bias then
     subtracts cost[x_i][k] (u8 saturating).  Leaving at any cell gives
-    E = cell, J = E - tec.  Returns 255 if any cell reaches 255 - bias."""
+    E = cell, J = E - tec.  Returns 255 if any cell reaches 255 - bias.
+    ``reenter=False`` drops the J entries (every segment from N): the pins use it only to
+    show that a case really chains a later segment through J."""
     M = cost.shape[1]
     L = len(dsq)
     best = [0, False]  # raw, overflow
@@ -52,7 +54,7 @@ def msv_brute(cost, bias, tbm, tec, tjb, dsq):
     def segments_from(row_min, J):
         for i in range(row_min, L + 1):
             entries = [u8(190 - tjb)]
-            if J is not None:
+            if J is not None and reenter:
                 entries.append(u8(J - tjb))
             for k in range(1, M + 1):
                 for entry in entries:
