@@ -152,6 +152,7 @@ struct hmg_profile {
   int vit_W = 0;                    // >0: block-per-sequence kernel vit_cta_kernel<W, Q> (Q = vit_Q)
   int pair_G = 0, pair_Q = 0;       // >0: s16x2 pair kernel vit_pair_kernel<G, Q> first, the above re-scores
   bool pair_scan = false;           // pair kernel: max-plus scan Lazy-F (G = 32 only; HMG_VIT_SCAN)
+  int pair_SG2 = 0;                 // >0: W = 2 without the per-row barrier, vit_cpair2_kernel<pair_Q, pair_SG2>
   int pair_W = 0, pair_SG = 1;      // >0: block pair kernel vit_cpair_kernel<pair_W, pair_Q, pair_SG>
                                     //     (pair_G = 32 W; pair_SG sequences per block share its table)
   int tbm_min = 0, rmax = 0;        // pair kernel window: min_k tBM_k, max(0, max_{x,k} rsc)
@@ -230,6 +231,9 @@ cudaError_t launch_vit_pair(int G, int Q, bool scan, const VitArgs& a, cudaStrea
 cudaError_t launch_vit_cpair(int W, int SG, int Q, const VitArgs& a, cudaStream_t st, int* ok);
 size_t vit_cpair_smem(int W, int SG, int Q);
 bool vit_cpair_available(int W, int SG, int Q);
+cudaError_t launch_vit_cpair2(int SG, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+size_t vit_cpair2_smem(int SG, int Q);
+bool vit_cpair2_available(int SG, int Q);
 int vit_pair_q_max();
 size_t vit_cta_smem(int W, int Q);
 int long_msv_q(int M);

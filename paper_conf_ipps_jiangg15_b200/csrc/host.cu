@@ -639,7 +639,9 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     b.redo_list = redo;
     b.redo_count = ctr + 1;
     int ok = 0;
-    if (p->pair_W > 0) {
+    if (p->pair_SG2 > 0) {
+      if ((e = launch_vit_cpair2(p->pair_SG2, p->pair_Q, b, st, &ok))) return cuda_status(e);
+    } else if (p->pair_W > 0) {
       if ((e = launch_vit_cpair(p->pair_W, p->pair_SG, p->pair_Q, b, st, &ok))) return cuda_status(e);
     } else {
       if ((e = launch_vit_pair(p->pair_G, p->pair_Q, p->pair_scan, b, st, &ok))) return cuda_status(e);
@@ -905,6 +907,10 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
           p->pair_G = 32 * W;
           p->pair_Q = qq;
         }
+        // two warps: the kernel without a per-row barrier (vit_cpair2.cuh) unless asked otherwise
+        const int sg2 = env_int("HMG_VIT_CPAIR2_SG", 2);
+        if (p->pair_W == 2 && sg2 > 0 && vit_cpair2_available(sg2, qq) && vit_cpair2_smem(sg2, qq) <= (size_t)smax)
+          p->pair_SG2 = sg2;
       }
     }
   }

@@ -500,11 +500,15 @@ def test_pipeline_many_survivors(M):
 
 
 @pytest.mark.parametrize("M", [2, 3, 64, 300, 513, 1024, 1025, 1500, 2048, 2600, 4000])
-@pytest.mark.parametrize("W", [2, 4, 8, 16])
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b"])
 def test_vit_block_pair_kernel(M, W, monkeypatch):
     """Block-per-sequence pair kernel (W warps per row, 2 cells per register, closed-form carries
-    across virtual warps); forced for small M with HMG_VIT_PAIR_CTA, used by default above 1024."""
+    across virtual warps); forced for small M with HMG_VIT_PAIR_CTA, used by default above 1024.
+    W = 2 runs the kernel without a per-row barrier (vit_cpair2.cuh); "2b" the barrier kernel."""
     monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
+    if W == "2b":
+        monkeypatch.setenv("HMG_VIT_CPAIR2_SG", "0")
+        W = 2
     monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
     rng = np.random.default_rng(M * 7 + W)
     for dd in [(7.0, 3.0), (1.0, 9.0)]:
@@ -517,11 +521,14 @@ def test_vit_block_pair_kernel(M, W, monkeypatch):
         assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)), dd
 
 
-@pytest.mark.parametrize("W", [2, 4, 8, 16])
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b"])
 def test_vit_block_pair_delete_chains_and_exits(W, monkeypatch):
     """D->D chains across every virtual-warp boundary (low halves -> high halves), strong hits that
     re-base the window or overflow, and gap-only sequences handed to the s32 kernel."""
     monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
+    if W == "2b":
+        monkeypatch.setenv("HMG_VIT_CPAIR2_SG", "0")
+        W = 2
     monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
     for M in (40, 700, 2000):
         rng = np.random.default_rng(M + W)
