@@ -118,6 +118,14 @@ void hmg_profile_destroy(hmg_profile* p);
  * immutable: create the searching profile with the returned parameters. */
 hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, double lambda, hmg_evparams* out);
 
+/* The same fit over a caller-supplied background database: every sequence of db is
+ * scored with the library's MSV and Viterbi-filter kernels on the profile's device, converted to
+ * bits with its own length (nats as hmg_msv_nats / hmg_vit_nats, null1 of its L), and
+ * mu = -ln(mean over finite scores of exp(-lambda * bits)) / lambda.  hmg_calibrate is this call
+ * on its generated sample.  db must live on the profile's device and hold >= 1 sequence; lambda
+ * > 0; the profile needs tsc.  Synchronous.  HMG_EINVAL on bad arguments, HMG_ECUDA. */
+hmg_status hmg_calibrate_db(const hmg_profile* p, const hmg_db* db, double lambda, hmg_evparams* out);
+
 
 /* ---------------------------------------------------------------- database */
 
@@ -236,6 +244,30 @@ hmg_status hmg_pipeline_batch(const hmg_profile* const* profs, int nprof, const 
                               void* stream, uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags,
                               int32_t* survivor_ids, int64_t* n_survivors, float* fwd_nats, int32_t* fwd_ids,
                               int64_t* n_fwd);
+
+/* Pass thresholds (reading R25) are integer tables by target length, built on the
+ * host from the profile's Gumbel parameters per F.  A compute call builds the tables it needs on
+ * first use (host binary search, cudaMalloc + cudaMemcpy: not allowed inside CUDA stream capture,
+ * where such a call returns HMG_EUNSUPPORTED and leaves the capture intact).  This call builds them
+ * ahead for MSV threshold F1 and Viterbi threshold F2 and target lengths up to Lmax (at least
+ * 40000), so that a later call -- e.g. one captured in a CUDA graph -- finds them.  Tables stay
+ * allocated until hmg_profile_destroy (graphs and other streams may hold them).
+ * Needs a device profile with ev; F in (0, 1]; Lmax >= 1. */
+hmg_status hmg_prepare_thresholds(const hmg_profile* p, double F1, double F2, int Lmax);
+
+/* ---------------------------------------------------------------- tuning (performance only) */
+
+/* Process-wide overrides of the kernel-geometry and schedule choices (the
+ * defaults are the measured ones).  The library never reads the environment: results never depend
+ * on these knobs (every kernel is exact), only performance does, and tests / sweeps set them here.
+ * Knobs (int): MSV_G, VIT_G, MSV_LLONG, NO_LONG_LANE, FWD_QMAX, FWD_W, FWD_S, VIT_CTA, VIT_CTA_W,
+ * VIT_GENERIC, NO_VIT_PAIR, VIT_PAIR_G, VIT_PAIR_CTA, VIT_SCAN, VIT_PAIR_W, VIT_PAIR_SG,
+ * VIT_CPAIR2, LONG_S32, PIPE_LLONG, PIPE_CHUNK, UPLOAD_PARTS, UPLOAD_FIRST_PERMILLE, UPLOAD_GROW,
+ * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS.  Geometry knobs take effect at profile / DB
+ * creation, schedule knobs at the next call.  HMG_EINVAL for an unknown name. */
+hmg_status hmg_set_tuning(const char* name, int value);
+/* Remove one override (name) or all of them (name == NULL). */
+hmg_status hmg_clear_tuning(const char* name);
 
 /* ---------------------------------------------------------------- instrumentation */
 

@@ -21,7 +21,6 @@ constexpr int16_t kNegE = -16384;   // "minus infinity" emission / carry of the 
 constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
 
 // ---------------------------------------------------------------- MSV kernel arguments
-constexpr int kMaxGates = 12;   // = kUploadParts (host.cu)
 
 struct MsvArgs {
   const uint32_t* words;     // packed residues
@@ -39,11 +38,6 @@ struct MsvArgs {
   const int32_t* list;       // exact kernel: sorted indices to redo
   const int64_t* nlist;      // exact kernel: device count
   uint8_t* scratch;          // exact kernel: per-warp row buffers
-  // fast kernel, overlapped upload (hmg_pipeline_upload): the sorted range is in ngate parts,
-  // part q = [.., gate_end[q]); a batch waits until gate_flag[q] != 0 (set behind part q's H2D)
-  int ngate;
-  const unsigned* gate_flag;
-  long long gate_end[kMaxGates];
 };
 
 // Many-profile MSV (msv_multi.cuh): a bucket of profiles with one lane geometry
@@ -184,13 +178,16 @@ struct hmg_profile {
     uint32_t* d;
   };
   std::vector<Tab> msv_tabs;
-  // threshold caches (built on first use per F and DB Lmax)
+  // threshold tables (built on first use per F and length range, or by hmg_prepare_thresholds).
+  // Every table handed out stays allocated until hmg_profile_destroy: a CUDA graph captured with
+  // one, or a call still running on another stream, never sees it freed or replaced.
   std::mutex mu;
   struct Thr {
     double F = -1;
     int Lmax = -1;
     void* d = nullptr;
-  } thr_msv, thr_vit;
+  };
+  std::vector<Thr> thr_msv, thr_vit;
 };
 
 struct hmg_db {

@@ -12,9 +12,12 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
 #include <numeric>
 #include <random>
+#include <string>
 #include <vector>
 
 #include "hmg_internal.h"
@@ -169,9 +172,27 @@ hmg_status upload(T** d, const T* h, size_t n) {
   return cuda_status(e);
 }
 
-int env_int(const char* name, int dflt) {
-  const char* v = getenv(name);
-  return v ? atoi(v) : dflt;
+// Tuning / debug overrides (hmg_set_tuning): the library never reads the process environment.
+// Knob names are the kernel-geometry and schedule choices of DESIGN.md; an unset knob takes the
+// measured default at its call site.
+const char* const kTuneNames[] = {
+    "MSV_G", "VIT_G", "MSV_LLONG", "NO_LONG_LANE", "FWD_QMAX", "FWD_W", "FWD_S", "VIT_CTA", "VIT_CTA_W",
+    "VIT_GENERIC", "NO_VIT_PAIR", "VIT_PAIR_G", "VIT_PAIR_CTA", "VIT_SCAN", "VIT_PAIR_W", "VIT_PAIR_SG",
+    "VIT_CPAIR2", "LONG_S32", "PIPE_LLONG", "PIPE_CHUNK", "UPLOAD_PARTS", "UPLOAD_FIRST_PERMILLE",
+    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS"};
+std::mutex g_tune_mu;
+std::map<std::string, int> g_tune;
+
+bool tune_known(const char* name) {
+  for (const char* k : kTuneNames)
+    if (!strcmp(k, name)) return true;
+  return false;
+}
+
+int tune_int(const char* name, int dflt) {
+  std::lock_guard<std::mutex> g(g_tune_mu);
+  auto it = g_tune.find(name);
+  return it == g_tune.end() ? dflt : it->second;
 }
 
 // Stream-ordered scratch (Scratch below) comes from the device's default memory pool; its default
@@ -196,7 +217,7 @@ void keep_pool_cached(int device) {
 void msv_geometry(int M, int* G, int* Q) {
   // lane-group size from the G sweep on the config-2 DB (profiles/msv_sweep_r01.txt)
   int g = M < 80 ? 4 : M <= 450 ? 8 : M <= 640 ? 16 : 32;
-  const int o = env_int("HMG_MSV_G", 0);
+  const int o = tune_int("MSV_G", 0);
   if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
   // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
   // fast kernel records each cell's value in the cell it feeds (t_{i+1}[k+1]).
@@ -211,7 +232,7 @@ void msv_geometry(int M, int* G, int* Q) {
 
 void vit_geometry(int M, int* G, int* Q) {
   int g = M <= 128 ? 8 : M <= 256 ? 16 : 32;
-  const int o = env_int("HMG_VIT_G", 0);
+  const int o = tune_int("VIT_G", 0);
   if (o == 8 || o == 16 || o == 32) g = o;
   int q = (M + g - 1) / g;
   while (q > vit_q_max(g) && g < 32) {
@@ -226,7 +247,6 @@ void vit_geometry(int M, int* G, int* Q) {
 std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
   const int M = p.M;
   const int ROWW = Q * G;
-  std::vector<uint32_t> t((size_t)kRows * ROWW);
   const int n4 = Q / 4, r = Q % 4;
   auto word_index = [&](int z, int q) {
     if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
@@ -257,7 +277,6 @@ std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
           out[(size_t)k * (copy + 4 * G) + (size_t)x * stride + word_index(z, q)] =
               (uint32_t)lo | ((uint32_t)hi << 16);
         }
-  (void)t;
   return out;
 }
 
@@ -384,51 +403,53 @@ struct Scratch {
   }
 };
 
-// threshold tables, cached per (F, Lmax) in the profile
-hmg_status msv_thr_table(hmg_profile* p, const hmg_db* db, double F, const uint16_t** out) {
+// threshold tables, per (F, length range) in the profile; a table is never freed or replaced
+// while the profile lives (graphs and concurrent streams may hold its pointer).  Building one
+// (host binary search + cudaMalloc / cudaMemcpy) is not allowed under stream capture: a call being
+// captured finds its tables prepared (hmg_prepare_thresholds or an eager call) or fails with
+// HMG_EUNSUPPORTED without touching the capture.
+template <class T, class Fill>
+hmg_status thr_table(hmg_profile* p, std::vector<hmg_profile::Thr>& cache, int Lmax, double F, cudaStream_t st,
+                     Fill fill, const T** out) {
   std::lock_guard<std::mutex> g(p->mu);
-  auto& c = p->thr_msv;
-  if (c.d && c.F == F && c.Lmax >= db->Lmax) {
-    *out = (const uint16_t*)c.d;
-    return HMG_OK;
-  }
-  std::vector<uint16_t> h((size_t)db->Lmax + 1, 256);
-  const double mu = p->ev.mu_msv, lam = p->ev.lambda_msv;
-  for (int L = 1; L <= db->Lmax; ++L)
-    h[L] = (uint16_t)least_passing(0, 254, [&](int r) { return passes(msv_nats_of(r, L), L, mu, lam, F); });
-  if (c.d) cudaFree(c.d);
-  c.d = nullptr;
-  uint16_t* d = nullptr;
+  for (const auto& c : cache)
+    if (c.F == F && c.Lmax >= Lmax) {
+      *out = (const T*)c.d;
+      return HMG_OK;
+    }
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (st && cudaStreamIsCapturing(st, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+    return HMG_EUNSUPPORTED;
+  cudaGetLastError();
+  const int L1 = std::max(Lmax, 40000);            // one table covers every protein length seen so far
+  std::vector<T> h((size_t)L1 + 1);
+  fill(h, L1);
+  T* d = nullptr;
   hmg_status s = upload(&d, h.data(), h.size());
   if (s != HMG_OK) return s;
-  c.d = d;
-  c.F = F;
-  c.Lmax = db->Lmax;
+  cache.push_back({F, L1, d});
   *out = d;
   return HMG_OK;
 }
 
-hmg_status vit_thr_table(hmg_profile* p, const hmg_db* db, double F, const int32_t** out) {
-  std::lock_guard<std::mutex> g(p->mu);
-  auto& c = p->thr_vit;
-  if (c.d && c.F == F && c.Lmax >= db->Lmax) {
-    *out = (const int32_t*)c.d;
-    return HMG_OK;
-  }
-  std::vector<int32_t> h((size_t)db->Lmax + 1, 32767);
+hmg_status msv_thr_table(hmg_profile* p, const hmg_db* db, double F, const uint16_t** out, cudaStream_t st = nullptr,
+                         int Lmax = -1) {
+  const double mu = p->ev.mu_msv, lam = p->ev.lambda_msv;
+  return thr_table<uint16_t>(p, p->thr_msv, Lmax >= 0 ? Lmax : db->Lmax, F, st, [&](std::vector<uint16_t>& h, int L1) {
+    h[0] = 256;
+    for (int L = 1; L <= L1; ++L)
+      h[L] = (uint16_t)least_passing(0, 254, [&](int r) { return passes(msv_nats_of(r, L), L, mu, lam, F); });
+  }, out);
+}
+
+hmg_status vit_thr_table(hmg_profile* p, const hmg_db* db, double F, const int32_t** out, cudaStream_t st = nullptr,
+                         int Lmax = -1) {
   const double mu = p->ev.mu_vit, lam = p->ev.lambda_vit;
-  for (int L = 1; L <= db->Lmax; ++L)
-    h[L] = least_passing(-32768, 32766, [&](int r) { return passes(vit_nats_of(r, L), L, mu, lam, F); });
-  if (c.d) cudaFree(c.d);
-  c.d = nullptr;
-  int32_t* d = nullptr;
-  hmg_status s = upload(&d, h.data(), h.size());
-  if (s != HMG_OK) return s;
-  c.d = d;
-  c.F = F;
-  c.Lmax = db->Lmax;
-  *out = d;
-  return HMG_OK;
+  return thr_table<int32_t>(p, p->thr_vit, Lmax >= 0 ? Lmax : db->Lmax, F, st, [&](std::vector<int32_t>& h, int L1) {
+    h[0] = 32767;
+    for (int L = 1; L <= L1; ++L)
+      h[L] = least_passing(-32768, 32766, [&](int r) { return passes(vit_nats_of(r, L), L, mu, lam, F); });
+  }, out);
 }
 
 MsvArgs msv_args(const hmg_profile* p, const hmg_db* db) {
@@ -459,21 +480,17 @@ double mean_len(const hmg_db* db) { return db->nseq ? (double)db->residues / (do
 // first pipe_nlong sequences are scored by the pipeline long lane instead.
 hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S,
                         int64_t pipe_nlong, bool pdl = false, bool mark0 = true,
-                        unsigned long long* ctr_zeroed = nullptr, int64_t end = -1,
-                        int ngate = 0, const unsigned* gate_flag = nullptr, const int64_t* gate_end = nullptr) {
+                        unsigned long long* ctr_zeroed = nullptr, int64_t end = -1) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
   MsvArgs a = msv_args(p, db);
   a.raw = raw_sorted;
-  a.ngate = ngate;
-  a.gate_flag = gate_flag;
-  for (int q = 0; q < ngate && q < kMaxGates; ++q) a.gate_end[q] = gate_end[q];
   if (end >= 0) a.nseq = end;          // sorted range [pipe_nlong, end) only (overlapped upload)
   if (pipe_nlong >= 0) {
     a.nlong = pipe_nlong;
     a.skip_long = 1;
   } else {  // in-kernel whole-warp queue: L > max(1000, 8 x mean length) (env HMG_MSV_LLONG)
-    a.nlong = count_longer(db, env_int("HMG_MSV_LLONG", (int)std::max(1000.0, 8.0 * mean_len(db))));
+    a.nlong = count_longer(db, tune_int("MSV_LLONG", (int)std::max(1000.0, 8.0 * mean_len(db))));
     a.skip_long = 0;
   }
   // (with pdl the counters must be zeroed before the preceding kernel: any stream operation
@@ -535,7 +552,7 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
 hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
   int64_t nlong = -1;
   mark(0, st);
-  if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && db->nlong > 0 && !env_int("HMG_NO_LONG_LANE", 0)) {
+  if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && db->nlong > 0 && !tune_int("NO_LONG_LANE", 0)) {
     LongArgs la{};
     hmg_status s = run_msv_long_chunks(p, db, st, raw_sorted, S, &la);
     if (s != HMG_OK) return s;
@@ -687,6 +704,38 @@ const char* hmg_strerror(hmg_status s) {
 
 int64_t hmg_kernel_launches(void) { return g_launches.load(); }
 
+hmg_status hmg_set_tuning(const char* name, int value) {
+  if (!name || !tune_known(name)) return HMG_EINVAL;
+  std::lock_guard<std::mutex> g(g_tune_mu);
+  g_tune[name] = value;
+  return HMG_OK;
+}
+
+hmg_status hmg_clear_tuning(const char* name) {
+  std::lock_guard<std::mutex> g(g_tune_mu);
+  if (!name) {
+    g_tune.clear();
+    return HMG_OK;
+  }
+  if (!tune_known(name)) return HMG_EINVAL;
+  g_tune.erase(name);
+  return HMG_OK;
+}
+
+hmg_status hmg_prepare_thresholds(const hmg_profile* pc, double F1, double F2, int Lmax) {
+  hmg_profile* p = const_cast<hmg_profile*>(pc);
+  if (!p || !p->has_ev || p->device < 0 || Lmax < 1 || !(F1 > 0.0 && F1 <= 1.0) || !(F2 > 0.0 && F2 <= 1.0))
+    return HMG_EINVAL;
+  Dev dg(p->device);
+  const uint16_t* tm = nullptr;
+  hmg_status s = msv_thr_table(p, nullptr, F1, &tm, nullptr, Lmax);
+  if (s == HMG_OK && p->has_tsc) {
+    const int32_t* tv = nullptr;
+    s = vit_thr_table(p, nullptr, F2, &tv, nullptr, Lmax);
+  }
+  return s;
+}
+
 hmg_status hmg_set_stage_timing(int enable) {
   std::lock_guard<std::mutex> g(g_timer_mu);
   if (enable && !g_timer.on) {
@@ -805,9 +854,9 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   p->msc_max = -INFINITY;
   for (size_t i = 0; i < (size_t)M * kAlpha; ++i) p->msc_max = std::max(p->msc_max, msc[i]);
   // ---- Forward stage geometry (forward.cu): emission rows staged in shared memory as fit
-  const int fwd_qmax = env_int("HMG_FWD_QMAX", 16) >= 16 ? 16 : 8;   // 16: profiles/fwd_bench_r01e.jsonl
+  const int fwd_qmax = tune_int("FWD_QMAX", 16) >= 16 ? 16 : 8;   // 16: profiles/fwd_bench_r01e.jsonl
   if (tsc && (fwd_geometry(M, &p->fwd_T, &p->fwd_Q, fwd_qmax) || fwd_geometry(M, &p->fwd_T, &p->fwd_Q, 8))) {
-    const int wo = env_int("HMG_FWD_W", 0);   // whole warps per sequence (1 = no sub-warp groups)
+    const int wo = tune_int("FWD_W", 0);   // whole warps per sequence (1 = no sub-warp groups)
     if (wo == 1 || wo == 2 || wo == 4 || wo == 8 || wo == 16) {
       int q = 2;
       while (32 * wo * q < M && q < 16) q *= 2;
@@ -826,7 +875,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     if (device >= 0) {
       Dev dg(device);
       p->fwd_S = fwd_pick_s(p->fwd_T, p->fwd_Q, rows);
-      const int so = env_int("HMG_FWD_S", 0);
+      const int so = tune_int("FWD_S", 0);
       if (so > 0) p->fwd_S = so;
       if (p->fwd_S == 0) p->fwd_W = p->fwd_T = 0;   // no launchable configuration: Forward unsupported
     }
@@ -836,9 +885,9 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   msv_geometry(M, &p->msv_G, &p->msv_Q);
   if (tsc) {
     vit_geometry(M, &p->vit_G, &p->vit_Q);
-    if (p->vit_Q == 0 || env_int("HMG_VIT_CTA", 0)) {   // long models: block-per-sequence kernel
+    if (p->vit_Q == 0 || tune_int("VIT_CTA", 0)) {   // long models: block-per-sequence kernel
       int W = M <= 2048 ? 8 : 16;           // W = 8 keeps two 256-thread blocks per SM up to M = 2048
-      const int wo = env_int("HMG_VIT_CTA_W", 0);
+      const int wo = tune_int("VIT_CTA_W", 0);
       if (wo == 4 || wo == 8 || wo == 16) W = wo;
       int Q = (M + 32 * W - 1) / (32 * W);
       Q += Q & 1;
@@ -853,7 +902,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
         p->vit_Q = 0;
       }
     }
-    p->vit_generic = p->vit_Q == 0 || env_int("HMG_VIT_GENERIC", 0);
+    p->vit_generic = p->vit_Q == 0 || tune_int("VIT_GENERIC", 0);
     // s16x2 pair kernel (vit_pair.cuh) in front of the s32 kernels: its 16-bit window must hold
     // xN + move(L) + tBM_k .. 32767 for typical L, so entry scores and emissions must be moderate
     int tmin = 32767, rmx = 0;
@@ -861,18 +910,18 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     for (int16_t v : p->rsc) rmx = std::max(rmx, (int)v);
     p->tbm_min = tmin;
     p->rmax = rmx;
-    if (tmin > -16384 && rmx < 8192 && !env_int("HMG_NO_VIT_PAIR", 0)) {
+    if (tmin > -16384 && rmx < 8192 && !tune_int("NO_VIT_PAIR", 0)) {
       // lane-group size from the sweep (profiles/vit_pair_sweep_r01.jsonl): registers per lane
       // (12 Q + ~30) set the warps per SM, so small Q (4-8) wins over fewer lanes per sequence
       int g = M <= 64 ? 8 : M <= 128 ? 16 : 32;
-      const int o = env_int("HMG_VIT_PAIR_G", 0);
+      const int o = tune_int("VIT_PAIR_G", 0);
       if (o == 8 || o == 16 || o == 32) g = o;
       int q = (M + 2 * g - 1) / (2 * g);
       while (q > vit_pair_q_max() && g < 32) {
         g *= 2;
         q = (M + 2 * g - 1) / (2 * g);
       }
-      if (q <= vit_pair_q_max() && !env_int("HMG_VIT_PAIR_CTA", 0)) {
+      if (q <= vit_pair_q_max() && !tune_int("VIT_PAIR_CTA", 0)) {
         p->pair_G = g;
         p->pair_Q = q;
         // Lazy-F by max-plus scan (f1) when D->D chains are long: its cost does not depend on the
@@ -880,18 +929,18 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
         double pdd = 0.0;
         for (int k = 0; k + 1 < M; ++k) pdd += std::exp((double)tsc[(size_t)k * 8 + 7]);
         pdd = M > 1 ? pdd / (M - 1) : 0.0;
-        p->pair_scan = g == 32 && env_int("HMG_VIT_SCAN", pdd > 0.6 ? 1 : 0);
+        p->pair_scan = g == 32 && tune_int("VIT_SCAN", pdd > 0.6 ? 1 : 0);
       } else {   // long models: block-per-sequence pair kernel, W warps on one DP row
         // W warps per sequence and SG sequences per block from the sweep on the config-4 shape
         // (profiles/vit_cpair_sweep_r01.jsonl): 2 warps x 16 registers per thread, 2 sequences
         // per block sharing the table, up to M = 2048; wider rows above
         int W = M <= 2048 ? 2 : 4, SG = M <= 2048 ? 2 : 1;
-        const int wo = env_int("HMG_VIT_PAIR_W", 0);
+        const int wo = tune_int("VIT_PAIR_W", 0);
         if (wo == 2 || wo == 4 || wo == 8 || wo == 16) {
           W = wo;
           SG = W == 2 ? 2 : W == 4 ? 3 : W == 8 ? 2 : 1;
         }
-        SG = env_int("HMG_VIT_PAIR_SG", SG);
+        SG = tune_int("VIT_PAIR_SG", SG);
         int qq = std::max(2, (M + 64 * W - 1) / (64 * W));
         while (!vit_cpair_available(W, SG, qq) && W < 16) {   // models too long for W warps
           W *= 2;
@@ -908,7 +957,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
           p->pair_Q = qq;
         }
         // two warps: the kernel without a per-row barrier (vit_cpair2.cuh) unless asked otherwise
-        const int sg2 = env_int("HMG_VIT_CPAIR2_SG", 2);
+        const int sg2 = tune_int("VIT_CPAIR2", 2);
         if (p->pair_W == 2 && sg2 > 0 && vit_cpair2_available(sg2, qq) && vit_cpair2_smem(sg2, qq) <= (size_t)smax)
           p->pair_SG2 = sg2;
       }
@@ -968,8 +1017,8 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   }
   // pipeline long lane: whole-warp Viterbi with the pair lane (the pair tables when G = 32, models
   // up to 1024 nodes) or the s32 latency lane (models up to 512 nodes)
-  const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !env_int("HMG_LONG_S32", 0);
-  if (st == HMG_OK && tsc && (lpair || M <= 512) && !env_int("HMG_NO_LONG_LANE", 0)) {
+  const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !tune_int("LONG_S32", 0);
+  if (st == HMG_OK && tsc && (lpair || M <= 512) && !tune_int("NO_LONG_LANE", 0)) {
     const int QL = long_msv_q(M);
     auto tm = msv_table(*p, 32, QL);
     st = upload(&p->d_long_msv, tm.data(), tm.size());
@@ -1007,6 +1056,54 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   return HMG_OK;
 }
 
+hmg_status hmg_calibrate_db(const hmg_profile* p, const hmg_db* db, double lambda, hmg_evparams* out) {
+  if (!p || !db || !out || !(lambda > 0) || !p->has_tsc || p->device < 0 || db->device != p->device ||
+      db->nseq < 1)
+    return HMG_EINVAL;
+  const int64_t n = db->nseq;
+  Dev dg(p->device);
+  uint8_t* d_m = nullptr;
+  int16_t* d_v = nullptr;
+  hmg_status s = HMG_OK;
+  cudaError_t e = cudaMalloc(&d_m, (size_t)n);
+  if (e == cudaSuccess) e = cudaMalloc(&d_v, sizeof(int16_t) * (size_t)n);
+  if (e == cudaSuccess) {
+    s = hmg_msv(p, db, 0.02, nullptr, d_m, nullptr);
+    if (s == HMG_OK) s = hmg_viterbi(p, db, nullptr, 0, 1e-3, nullptr, d_v, nullptr);
+  } else {
+    s = cuda_status(e);
+  }
+  std::vector<uint8_t> hm((size_t)n);
+  std::vector<int16_t> hv((size_t)n);
+  if (s == HMG_OK) {
+    e = cudaMemcpy(hm.data(), d_m, (size_t)n, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(hv.data(), d_v, sizeof(int16_t) * (size_t)n, cudaMemcpyDeviceToHost);
+    s = cuda_status(e);
+  }
+  cudaFree(d_m);
+  cudaFree(d_v);
+  if (s != HMG_OK) return s;
+  std::vector<int> len((size_t)n);                 // caller-order lengths
+  for (int64_t j = 0; j < n; ++j) len[(size_t)db->order[(size_t)j]] = db->len_sorted[(size_t)j];
+  // closed-form ML location of a Gumbel with known lambda over the finite bit scores
+  auto fit = [&](auto nats_of, const auto& raw) {
+    double acc = 0;
+    int64_t cnt = 0;
+    for (int64_t j = 0; j < n; ++j) {
+      const int L = len[(size_t)j];
+      const float nats = nats_of((int)raw[(size_t)j], L);
+      if (!std::isfinite(nats)) continue;
+      acc += exp(-lambda * ((double)(nats - null1_of(L)) / kLn2));
+      ++cnt;
+    }
+    return cnt ? -log(acc / (double)cnt) / lambda : 0.0;
+  };
+  out->mu_msv = fit(msv_nats_of, hm);
+  out->mu_vit = fit(vit_nats_of, hv);
+  out->lambda_msv = out->lambda_vit = lambda;
+  return HMG_OK;
+}
+
 hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, double lambda, hmg_evparams* out) {
   if (!p || !out || n < 1 || L < 1 || !(lambda > 0) || !p->has_tsc || p->device < 0) return HMG_EINVAL;
   // HMMER3 amino background (reading R34) and 0.05% X, as the synthetic databases
@@ -1030,44 +1127,9 @@ hmg_status hmg_calibrate(const hmg_profile* p, int n, int L, uint64_t seed, doub
   hmg_db* db = nullptr;
   hmg_status s = hmg_db_create(dsq.data(), off.data(), n, p->device, &db);
   if (s != HMG_OK) return s;
-  Dev dg(p->device);
-  uint8_t* d_m = nullptr;
-  int16_t* d_v = nullptr;
-  cudaError_t e = cudaMalloc(&d_m, (size_t)n);
-  if (e == cudaSuccess) e = cudaMalloc(&d_v, sizeof(int16_t) * (size_t)n);
-  if (e == cudaSuccess) {
-    s = hmg_msv(p, db, 0.02, nullptr, d_m, nullptr);
-    if (s == HMG_OK) s = hmg_viterbi(p, db, nullptr, 0, 1e-3, nullptr, d_v, nullptr);
-  } else {
-    s = cuda_status(e);
-  }
-  std::vector<uint8_t> hm((size_t)n);
-  std::vector<int16_t> hv((size_t)n);
-  if (s == HMG_OK) {
-    e = cudaMemcpy(hm.data(), d_m, (size_t)n, cudaMemcpyDeviceToHost);
-    if (e == cudaSuccess) e = cudaMemcpy(hv.data(), d_v, sizeof(int16_t) * (size_t)n, cudaMemcpyDeviceToHost);
-    s = cuda_status(e);
-  }
-  cudaFree(d_m);
-  cudaFree(d_v);
+  s = hmg_calibrate_db(p, db, lambda, out);
   hmg_db_destroy(db);
-  if (s != HMG_OK) return s;
-  const float null = null1_of(L);
-  auto fit = [&](auto nats_of, const auto& raw) {
-    double acc = 0;
-    int cnt = 0;
-    for (auto r : raw) {
-      const float nats = nats_of((int)r, L);
-      if (!std::isfinite(nats)) continue;
-      acc += exp(-lambda * ((double)(nats - null) / kLn2));
-      ++cnt;
-    }
-    return cnt ? -log(acc / cnt) / lambda : 0.0;
-  };
-  out->mu_msv = fit(msv_nats_of, hm);
-  out->mu_vit = fit(vit_nats_of, hv);
-  out->lambda_msv = out->lambda_vit = lambda;
-  return HMG_OK;
+  return s;
 }
 
 hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
@@ -1117,8 +1179,8 @@ void hmg_profile_destroy(hmg_profile* p) {
     cudaFree(p->d_fwd_t);
     cudaFree(p->d_fwd_c);
     for (auto& t : p->msv_tabs) cudaFree(t.d);
-    cudaFree(p->thr_msv.d);
-    cudaFree(p->thr_vit.d);
+    for (auto& t : p->thr_msv) cudaFree(t.d);
+    for (auto& t : p->thr_vit) cudaFree(t.d);
     cudaGetLastError();
   }
   delete p;
@@ -1203,8 +1265,8 @@ hmg_status hmg_db_create(const uint8_t* dsq, const int64_t* off, int64_t nseq, i
   std::vector<int32_t> cstart(1, 0);
   {
     const double mean = nseq ? (double)res / (double)nseq : 0.0;
-    db->long_cut = env_int("HMG_PIPE_LLONG", (int)std::max(1500.0, 8.0 * mean));
-    db->chunk_rows = std::max(6, env_int("HMG_PIPE_CHUNK", 1032) / 6 * 6);
+    db->long_cut = tune_int("PIPE_LLONG", (int)std::max(1500.0, 8.0 * mean));
+    db->chunk_rows = std::max(6, tune_int("PIPE_CHUNK", 1032) / 6 * 6);
     while (db->nlong < nseq && db->len_sorted[db->nlong] > db->long_cut) {
       const int L = db->len_sorted[db->nlong];
       cstart.push_back(cstart.back() + (L + db->chunk_rows - 1) / db->chunk_rows);
@@ -1297,7 +1359,7 @@ hmg_status hmg_msv(const hmg_profile* pc, const hmg_db* db, double F1, void* str
   cudaStream_t st = (cudaStream_t)stream;
   const uint16_t* thr = nullptr;
   if (pass) {
-    hmg_status s = msv_thr_table(p, db, F1, &thr);
+    hmg_status s = msv_thr_table(p, db, F1, &thr, st);
     if (s != HMG_OK) return s;
   }
   cudaError_t e = cudaSuccess;
@@ -1330,7 +1392,7 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
   cudaStream_t st = (cudaStream_t)stream;
   const int32_t* thr = nullptr;
   if (pass) {
-    hmg_status s = vit_thr_table(p, db, F2, &thr);
+    hmg_status s = vit_thr_table(p, db, F2, &thr, st);
     if (s != HMG_OK) return s;
   }
   cudaError_t e = cudaSuccess;
@@ -1363,27 +1425,34 @@ hmg_status hmg_viterbi(const hmg_profile* pc, const hmg_db* db, const int32_t* i
 
 static cudaStream_t* side_streams(int device);
 
-// The overlapped upload marks each part as landed by a 4-byte H2D copy of the value 1 into a
-// device flag, queued on the copy stream right behind the part (the copy engine completes copies
-// of a stream in order), which the single gated MSV launch polls.  Source: one pinned word.
-static const unsigned* pinned_one() {
-  static unsigned* one = [] {
-    unsigned* h = nullptr;
-    if (cudaHostAlloc(&h, sizeof(unsigned), cudaHostAllocPortable) != cudaSuccess) {
-      cudaGetLastError();
-      return (unsigned*)nullptr;
-    }
-    *h = 1u;
-    return h;
-  }();
-  return one;
-}
-
 // h_image (optional): pinned host copy of the packed DB image (hmg_db_image); it is uploaded in
 // kUploadParts length-ordered parts on a side stream while the MSV kernel scores the parts that
 // have landed (one launch per part), so the H2D overlaps the filter.
-constexpr int kUploadParts = 12;    // capacity; parts used: HMG_UPLOAD_PARTS (default 6)
-static_assert(kUploadParts <= kMaxGates, "one landing gate per upload part");
+constexpr int kUploadParts = 12;    // capacity; parts used: tuning UPLOAD_PARTS (default 6)
+
+// Joins side streams back into the caller's stream on every exit path of a call that forked
+// them (declared after the call's Scratch, so it runs first and the scratch is freed on `st`
+// only after the side-stream work that uses it), and destroys the call's events.
+struct SideJoin {
+  cudaStream_t st;
+  std::vector<cudaStream_t> side;
+  std::vector<cudaEvent_t> events;
+  explicit SideJoin(cudaStream_t s) : st(s) {}
+  void add(cudaStream_t s) {
+    if (s && s != st && std::find(side.begin(), side.end(), s) == side.end()) side.push_back(s);
+  }
+  ~SideJoin() {
+    for (cudaStream_t s : side) {
+      cudaEvent_t ev = nullptr;
+      if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess) {
+        if (cudaEventRecord(ev, s) == cudaSuccess) cudaStreamWaitEvent(st, ev, 0);
+        cudaEventDestroy(ev);
+      }
+    }
+    for (cudaEvent_t ev : events)
+      if (ev) cudaEventDestroy(ev);
+  }
+};
 
 static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double F1, double F2, void* stream,
                                 uint8_t* msv_raw, int16_t* vit_raw, uint8_t* flags, int32_t* survivor_ids,
@@ -1397,8 +1466,8 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
   if (db->nseq == 0) return n_survivors ? cuda_status(set_count(n_survivors, 0, st)) : HMG_OK;
   const uint16_t* tm = nullptr;
   const int32_t* tv = nullptr;
-  hmg_status s = msv_thr_table(p, db, F1, &tm);
-  if (s == HMG_OK) s = vit_thr_table(p, db, F2, &tv);
+  hmg_status s = msv_thr_table(p, db, F1, &tm, st);
+  if (s == HMG_OK) s = vit_thr_table(p, db, F2, &tv, st);
   if (s != HMG_OK) return s;
   cudaError_t e = cudaSuccess;
   {
@@ -1415,14 +1484,12 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     // (programmatic dependent launch) fills the other SMs
     const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 &&
                            (p->long_pair || (!p->vit_generic && p->vit_W == 0)) &&
-                           !env_int("HMG_NO_LONG_LANE", 0)) ? db->nlong : 0;
+                           !tune_int("NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
-    // part counters (2 per part) + the gated launch's landing flags (u32, one per part)
-    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 3 * kUploadParts, &e);
+    // work-queue counters (2 per upload part)
+    auto* mctr = (unsigned long long*)S.get(sizeof(unsigned long long) * 2 * kUploadParts, &e);
     if (e) return cuda_status(e);
-    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 3 * kUploadParts, st))) return cuda_status(e);
-    unsigned* gate_flag = reinterpret_cast<unsigned*>(mctr + 2 * kUploadParts);
-    const unsigned* one = h_image && env_int("HMG_UPLOAD_GATED", 0) ? pinned_one() : nullptr;
+    if ((e = cudaMemsetAsync(mctr, 0, sizeof(unsigned long long) * 2 * kUploadParts, st))) return cuda_status(e);
     // overlapped upload: part boundaries (sorted indices), part 0 >= the long lane; part k's
     // words are one contiguous run of the image
     int64_t bnd[kUploadParts + 1] = {0};
@@ -1430,15 +1497,16 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     bnd[1] = n;
     cudaEvent_t up_ev[kUploadParts] = {};
     cudaStream_t cs = nullptr;
+    SideJoin join(st);                              // every exit: side streams joined into st
     if (h_image) {
-      nparts = std::max(2, std::min(kUploadParts, env_int("HMG_UPLOAD_PARTS", 6)));   // profiles/upload_parts_r01.jsonl
+      nparts = std::max(2, std::min(kUploadParts, tune_int("UPLOAD_PARTS", 6)));   // profiles/upload_parts_r01.jsonl
       // a small first part (the filter waits for it; later parts land faster than MSV consumes
       // them), then equal parts of the rest
-      const int first_pm = env_int("HMG_UPLOAD_FIRST_PERMILLE", 50);   // profiles/upload_parts_r01b.jsonl
+      const int first_pm = tune_int("UPLOAD_FIRST_PERMILLE", 50);   // profiles/upload_parts_r01b.jsonl
       // the rest in parts whose sizes follow a geometric ratio HMG_UPLOAD_GROW / 1000 (1000 = equal
       // parts); a ratio below 1 shrinks the last parts, whose MSV cannot start before they land
       const int64_t r0 = db->residues * first_pm / 1000;
-      const double g = std::max(1, env_int("HMG_UPLOAD_GROW", 1000)) / 1000.0;
+      const double g = std::max(1, tune_int("UPLOAD_GROW", 1000)) / 1000.0;
       double cut[kUploadParts] = {0.0}, wsum = 0.0, wk = 1.0;
       for (int q = 1; q < nparts; ++q, wk *= g) wsum += wk;
       wk = 1.0;
@@ -1454,6 +1522,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       cudaStream_t* side = side_streams(db->device);
       if (!side) return HMG_ECUDA;
       cs = side[0];
+      join.add(cs);
       cudaEvent_t fork = nullptr;
       if ((e = cudaEventCreateWithFlags(&fork, cudaEventDisableTiming))) return cuda_status(e);
       if ((e = cudaEventRecord(fork, st)) || (e = cudaStreamWaitEvent(cs, fork, 0))) return cuda_status(e);
@@ -1463,11 +1532,10 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
         const int64_t w0 = bnd[q] < n ? (int64_t)db->woff16_h[bnd[q]] * 4 : nw_all;
         const int64_t w1 = bnd[q + 1] < n ? (int64_t)db->woff16_h[bnd[q + 1]] * 4 : nw_all;
         if ((e = cudaEventCreateWithFlags(&up_ev[q], cudaEventDisableTiming))) return cuda_status(e);
+        join.events.push_back(up_ev[q]);
         if (w1 > w0 && (e = cudaMemcpyAsync(db->d_words + w0, h_image + w0, (size_t)(w1 - w0) * 4,
                                             cudaMemcpyHostToDevice, cs)))
           return cuda_status(e);
-        if (one && (e = cudaMemcpyAsync(gate_flag + q, one, sizeof(unsigned), cudaMemcpyHostToDevice, cs)))
-          return cuda_status(e);                    // landing flag of part q, behind its data
         if ((e = cudaEventRecord(up_ev[q], cs))) return cuda_status(e);
       }
       if ((e = cudaStreamWaitEvent(st, up_ev[0], 0))) return cuda_status(e);
@@ -1483,11 +1551,13 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     }
     if (overlap) {
       ms = side_streams(db->device)[1];
+      join.add(ms);
       cudaEvent_t f2 = nullptr;
       if ((e = cudaEventCreateWithFlags(&f2, cudaEventDisableTiming))) return cuda_status(e);
       if ((e = cudaEventRecord(f2, st)) || (e = cudaStreamWaitEvent(ms, f2, 0))) return cuda_status(e);
       cudaEventDestroy(f2);
       if ((e = cudaEventCreateWithFlags(&ms_done, cudaEventDisableTiming))) return cuda_status(e);
+      join.events.push_back(ms_done);
     }
     mark(0, st);
     if (nlong > 0) {
@@ -1508,7 +1578,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       la.thr = tm;
       // blocks (SMs) for the long-survivor Viterbi: about one per 20 long sequences, 2..16
       int nb = (int)std::min<int64_t>(std::max<int64_t>((nlong + 19) / 20, 2), 16);
-      nb = env_int("HMG_PIPE_LONG_SMS", nb);
+      nb = tune_int("PIPE_LONG_SMS", nb);
       int ok = 0;
       if ((e = launch_pipe_long_vit(p->long_QV, p->long_pair, la, nb, st, &ok))) return cuda_status(e);
       if (!ok) return HMG_EUNSUPPORTED;
@@ -1517,17 +1587,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       s = run_msv_fast(p, db, st, raw_sorted, S, nlong > 0 ? nlong : -1, nlong > 0, false, mctr);   // Fig 1: MSV
       if (s != HMG_OK) return s;
     } else {
-      if (one) {       // one launch over every part: each batch waits on its part's landing flag
-        int64_t gend[kUploadParts];
-        for (int q = 0; q < nparts; ++q) gend[q] = bnd[q + 1];
-        if (nlong < n) {
-          s = run_msv_fast(p, db, ms, raw_sorted, S, nlong, false, false, mctr, n, nparts, gate_flag, gend);
-          if (s != HMG_OK) return s;
-        }
-        // join the copy stream (after the launch, which must not wait for the upload)
-        if ((e = cudaStreamWaitEvent(ms, up_ev[nparts - 1], 0))) return cuda_status(e);
-      }
-      for (int q = 0; q < nparts && !one; ++q) {  // else: MSV of each part once it has landed
+      for (int q = 0; q < nparts; ++q) {          // MSV of each part once it has landed
         if ((e = cudaStreamWaitEvent(ms, up_ev[q], 0))) return cuda_status(e);
         const int64_t lo = std::max(bnd[q], nlong), hi = bnd[q + 1];
         if (hi > lo) {
@@ -1536,10 +1596,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
         }
       }
       if ((e = cudaEventRecord(ms_done, ms)) || (e = cudaStreamWaitEvent(st, ms_done, 0))) return cuda_status(e);
-      cudaEventDestroy(ms_done);
     }
-    if (h_image)
-      for (int q = 0; q < nparts; ++q) cudaEventDestroy(up_ev[q]);
     s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;
     e = msv_finish(raw_sorted, db->d_len, db->d_order, n, tm, msv_raw, flags, surv, n_survivors, survivor_ids, tmp,
@@ -1762,7 +1819,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
   // (measured, profiles/batch_bench_r01.jsonl: padding pays on small DBs -- fewer, fuller
   //  launches -- and costs ~5% of cells on large ones, where every bucket fills the GPU anyway)
   const bool large = n >= 50000;
-  const int pad_pct = env_int("HMG_MSV_BATCH_PAD", large ? 0 : 20);
+  const int pad_pct = tune_int("MSV_BATCH_PAD", large ? 0 : 20);
   for (size_t j = 0; j < idx.size();) {
     int G = 0, Q = 0;
     msv_geometry(profs[idx[j]]->M, &G, &Q);
@@ -1791,7 +1848,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
     tbm[r] = p->tbm;
     Mmax = std::max(Mmax, p->M);
     if (pass || tail) {
-      hmg_status s = msv_thr_table(p, db, F1, &thr[r]);
+      hmg_status s = msv_thr_table(p, db, F1, &thr[r], st);
       if (s != HMG_OK) return s;
     }
   }
@@ -1863,7 +1920,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
       // chunk = R rounds of the block's 8 warps x 32/G sequences: large R keeps the item-boundary
       // idling of a block's warps small (large DBs), R = 4 measured best on config-1-sized DBs
       const int per_round = (32 / b.G) * 8;
-      const int R = env_int("HMG_MSV_BATCH_ROUNDS", large ? 16 : 4);
+      const int R = tune_int("MSV_BATCH_ROUNDS", large ? 16 : 4);
       m.chunk = per_round * R;
       m.nchunks = (n + m.chunk - 1) / m.chunk;
       m.counter = ctr + bi;
@@ -1919,7 +1976,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
         return cuda_status(e);
       std::vector<const int32_t*> tv(nprof);
       for (int r = 0; r < nprof; ++r) {
-        hmg_status s = vit_thr_table(const_cast<hmg_profile*>(profs[rows[r]]), db, tail->F2, &tv[r]);
+        hmg_status s = vit_thr_table(const_cast<hmg_profile*>(profs[rows[r]]), db, tail->F2, &tv[r], st);
         if (s != HMG_OK) return s;
       }
       const int ns = std::min(nprof, kSideStreams);

@@ -97,16 +97,6 @@ struct ResStream {
   }
 };
 
-// spin (bounded: ~2 s, never a hang) until a flag written by a stream memory operation is set
-__device__ __forceinline__ void gate_wait(const unsigned* f) {
-  for (int it = 0;; ++it) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
-    if (v != 0u || it > (1 << 22)) break;
-    __nanosleep(500);
-  }
-}
-
 __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
   int T = max(xJ, 189) + 4;
@@ -345,13 +335,6 @@ __device__ __forceinline__ void msv_fast_body(const MsvArgs& a) {
     if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);
     b = __shfl_sync(0xffffffffu, b, 0);
     if (first + (long long)b >= a.nseq) break;
-    if (a.ngate > 0) {                 // overlapped upload: wait until this batch's part has landed
-      const long long last = min(first + (long long)b + NG, (long long)a.nseq) - 1;
-      int q = 0;
-      while (q < a.ngate - 1 && last >= a.gate_end[q]) ++q;
-      if (lane == 0) gate_wait(a.gate_flag + q);
-      __syncwarp();
-    }
     msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
   }
 }

@@ -6,38 +6,44 @@
 
 namespace hmg {
 namespace {
-template <int SG, int Q, int QMAX>
-const void* pick2(int q) {
+template <int SG, int TSM, int Q, int QMAX>
+const void* pick2(int q, size_t* smem) {
   if constexpr (Q > QMAX) {
     return nullptr;
   } else {
-    if (q == Q) return reinterpret_cast<const void*>(&vit_cpair2_kernel<Q, SG>);
-    return pick2<SG, Q + 1, QMAX>(q);
+    if (q == Q) {
+      *smem = VitCP2Smem<Q, SG, TSM>::bytes;
+      return reinterpret_cast<const void*>(&vit_cpair2_kernel<Q, SG, TSM>);
+    }
+    return pick2<SG, TSM, Q + 1, QMAX>(q, smem);
   }
 }
-const void* cpair2_ptr(int SG, int Q) {
-  switch (SG) {
-    case 1: return pick2<1, 8, 16>(Q);
-    case 2: return pick2<2, 2, 16>(Q);
-    case 3: return pick2<3, 8, 16>(Q);
+// variant = 10 * TSM + SG (TSM 2: tMM, tIM, tMI, tII streamed from shared memory)
+const void* cpair2_ptr(int var, int Q, size_t* smem) {
+  switch (var) {
+    case 2: return pick2<2, 0, 2, 16>(Q, smem);
+    case 22: return pick2<2, 2, 2, 16>(Q, smem);
+    case 23: return pick2<3, 2, 8, 16>(Q, smem);
   }
   return nullptr;
 }
-size_t cpair2_smem(int SG, int Q) {
-  const size_t tab = (size_t)21 * Q * 64 * 4;
-  const size_t grp = sizeof(uint32_t) * ((Q * 64 + 16 + 2 + 2 + 3) / 4 * 4);
-  return tab + sizeof(uint32_t) * 4 + (size_t)SG * grp;
-}
 }  // namespace
 
-size_t vit_cpair2_smem(int SG, int Q) { return cpair2_ptr(SG, Q) ? cpair2_smem(SG, Q) : 0; }
-bool vit_cpair2_available(int SG, int Q) { return cpair2_ptr(SG, Q) != nullptr; }
+size_t vit_cpair2_smem(int var, int Q) {
+  size_t b = 0;
+  return cpair2_ptr(var, Q, &b) ? b : 0;
+}
+bool vit_cpair2_available(int var, int Q) {
+  size_t b = 0;
+  return cpair2_ptr(var, Q, &b) != nullptr;
+}
 
-cudaError_t launch_vit_cpair2(int SG, int Q, const VitArgs& a, cudaStream_t st, int* ok) {
-  const void* fn = cpair2_ptr(SG, Q);
+cudaError_t launch_vit_cpair2(int var, int Q, const VitArgs& a, cudaStream_t st, int* ok) {
+  size_t smem = 0;
+  const void* fn = cpair2_ptr(var, Q, &smem);
   *ok = fn != nullptr;
   if (!fn) return cudaSuccess;
-  const size_t smem = cpair2_smem(SG, Q);
+  const int SG = var % 10;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = 0, per = 0;

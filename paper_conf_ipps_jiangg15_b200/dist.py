@@ -14,8 +14,6 @@ torch.distributed for the collectives.  All scoring happens in libhmg.
 """
 from __future__ import annotations
 
-import math
-
 import numpy as np
 
 
@@ -52,37 +50,67 @@ def unpack_results(words: np.ndarray):
     return msv, vit, flags
 
 
-def gather(packed, survivor_ids, n_survivors, global_ids, world: int, group=None):
-    """All-gather per-sequence result words and survivor lists (global caller ids).
+class Gatherer:
+    """All-gather of per-sequence result words and survivor lists (global caller ids) with
+    static shapes: every buffer is allocated once, padded to the largest snake shard
+    (``shard_sizes``), so a step issues its collectives with no host synchronisation and no
+    allocation (it can sit inside a CUDA graph or a timed loop).
 
-    packed        : device int32 [n_local] (pack_results)
-    survivor_ids  : device int32 [>= n_local] local caller indices, schedule order
-    n_survivors   : device int64 [1]
-    global_ids    : device int64 [n_local] global caller index of each local sequence
-    Returns device tensors: words [world, nmax], gids [world, nmax], counts [world],
-    surv [world, nmax] (global ids, first counts[r] valid per row).
+    n_global   : sequences in the whole database; world / rank as torch.distributed
+    global_ids : device int64 [n_local] global caller index of each local sequence
+    exchange   : False builds the static buffers without any collective (one process playing
+                 every rank in turn: ``local`` gives the slices all_gather_into_tensor would
+                 concatenate in rank order -- the one-GPU proof of the sharded path)
     """
-    import torch
-    import torch.distributed as dist
-    n_local = packed.numel()
-    nmax_t = torch.tensor([n_local], dtype=torch.int64, device=packed.device)
-    dist.all_reduce(nmax_t, op=dist.ReduceOp.MAX, group=group)
-    nmax = int(nmax_t.item())
-    pad = torch.zeros(nmax, dtype=torch.int32, device=packed.device)
-    pad[:n_local] = packed
-    words = torch.empty(world * nmax, dtype=torch.int32, device=packed.device)
-    dist.all_gather_into_tensor(words, pad, group=group)
-    gid = torch.full((nmax,), -1, dtype=torch.int64, device=packed.device)
-    gid[:n_local] = global_ids
-    gids = torch.empty(world * nmax, dtype=torch.int64, device=packed.device)
-    dist.all_gather_into_tensor(gids, gid, group=group)
-    counts = torch.empty(world, dtype=torch.int64, device=packed.device)
-    dist.all_gather_into_tensor(counts, n_survivors.reshape(1), group=group)
-    sv = torch.full((nmax,), -1, dtype=torch.int64, device=packed.device)
-    sv[:n_local] = global_ids[survivor_ids[:n_local].to(torch.int64).clamp_(0, max(n_local - 1, 0))]
-    surv = torch.empty(world * nmax, dtype=torch.int64, device=packed.device)
-    dist.all_gather_into_tensor(surv, sv, group=group)
-    return words.view(world, nmax), gids.view(world, nmax), counts, surv.view(world, nmax)
+
+    def __init__(self, n_global: int, world: int, global_ids, group=None, exchange: bool = True):
+        import torch
+        import torch.distributed as dist
+        self.world, self.group = world, group
+        self.nmax = max(shard_sizes(n_global, world))
+        dev = global_ids.device
+        self.n_local = global_ids.numel()
+        self.gid_local = global_ids.to(torch.int64)
+        self.pad = torch.zeros(self.nmax, dtype=torch.int32, device=dev)
+        self.words = torch.empty(world * self.nmax, dtype=torch.int32, device=dev)
+        self.counts = torch.empty(world, dtype=torch.int64, device=dev)
+        self.sv = torch.full((self.nmax,), -1, dtype=torch.int64, device=dev)
+        self.surv = torch.empty(world * self.nmax, dtype=torch.int64, device=dev)
+        self.gid_pad = torch.full((self.nmax,), -1, dtype=torch.int64, device=dev)
+        self.gid_pad[:self.n_local] = self.gid_local
+        self.gids = torch.empty(world * self.nmax, dtype=torch.int64, device=dev)
+        self.exchange = exchange
+        if world > 1 and exchange:
+            dist.all_gather_into_tensor(self.gids, self.gid_pad, group=group)   # once: the shard map is static
+        else:
+            self.gids[:self.nmax].copy_(self.gid_pad)
+
+    def local(self, msv_raw, vit_raw, flags, survivor_ids, n_survivors):
+        """This rank's padded slices (device ops only): result words and global survivor ids."""
+        import torch
+        n = self.n_local
+        self.pad[:n] = pack_results(msv_raw[:n], vit_raw[:n], flags[:n])
+        ids = survivor_ids[:n].to(torch.int64).clamp_(0, max(n - 1, 0))
+        self.sv[:n] = self.gid_local[ids]
+        return self.pad, self.sv, n_survivors.reshape(1)
+
+    def __call__(self, msv_raw, vit_raw, flags, survivor_ids, n_survivors):
+        """Gather every rank's results; returns device views words [world, nmax],
+        gids [world, nmax], counts [world], surv [world, nmax] (first counts[r] valid)."""
+        import torch.distributed as dist
+        if not self.exchange:
+            raise RuntimeError("Gatherer(exchange=False) has no collective step")
+        pad, sv, ns = self.local(msv_raw, vit_raw, flags, survivor_ids, n_survivors)
+        if self.world > 1:
+            dist.all_gather_into_tensor(self.words, pad, group=self.group)
+            dist.all_gather_into_tensor(self.counts, ns, group=self.group)
+            dist.all_gather_into_tensor(self.surv, sv, group=self.group)
+        else:
+            self.words.copy_(pad)
+            self.counts.copy_(ns)
+            self.surv.copy_(sv)
+        return (self.words.view(self.world, self.nmax), self.gids.view(self.world, self.nmax), self.counts,
+                self.surv.view(self.world, self.nmax))
 
 
 def assemble(words, gids, counts, surv, n_global: int):
@@ -95,28 +123,3 @@ def assemble(words, gids, counts, surv, n_global: int):
     msv, vit, flags = unpack_results(out)
     sl = [np.asarray(surv)[r, :int(c)] for r, c in enumerate(np.asarray(counts))]
     return msv, vit, flags, sl
-
-
-def calibrate(msc, tsc, device: int = 0, n: int = 1000, L: int = 200, seed: int = 7):
-    """Gumbel location mu for lambda = ln 2 of both filters, fitted on ``n``
-    background sequences of length ``L`` scored by the GPU kernels themselves
-    (closed-form ML location for known lambda).  Returns the hmg_evparams tuple."""
-    import torch
-
-    from . import hmg, synth
-    cal = synth.Database(np.full(n, L, np.int32), seed=seed)
-    dsq, off = cal.materialize()
-    p = hmg.Profile(msc, tsc, device=device)
-    db = hmg.Database(dsq, off, device=device)
-    dev = torch.device("cuda", device)
-    mraw = torch.zeros(n, dtype=torch.uint8, device=dev)
-    vraw = torch.zeros(n, dtype=torch.int16, device=dev)
-    hmg.hmg_msv(p, db, mraw)
-    hmg.hmg_viterbi(p, db, vraw)
-    torch.cuda.synchronize(dev)
-    lam = math.log(2)
-    null = hmg.hmg_null1_nats(L)
-    mb = np.array([(hmg.hmg_msv_nats(int(r), L) - null) / lam for r in mraw.cpu().numpy()])
-    vb = np.array([(hmg.hmg_vit_nats(int(r), L) - null) / lam for r in vraw.cpu().numpy()])
-    mu = lambda x: float(-np.log(np.mean(np.exp(-lam * x[np.isfinite(x)]))) / lam)
-    return (mu(mb), lam, mu(vb), lam)

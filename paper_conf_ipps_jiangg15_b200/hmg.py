@@ -65,6 +65,10 @@ SIGNATURES = {
     "hmg_strerror": (ctypes.c_char_p, [c_int]),
     "hmg_kernel_launches": (c_i64, []),
     "hmg_calibrate": (c_int, [c_p, c_int, c_int, ctypes.c_uint64, c_d, c_p]),
+    "hmg_calibrate_db": (c_int, [c_p, c_p, c_d, c_p]),
+    "hmg_prepare_thresholds": (c_int, [c_p, c_d, c_d, c_int]),
+    "hmg_set_tuning": (c_int, [ctypes.c_char_p, c_int]),
+    "hmg_clear_tuning": (c_int, [ctypes.c_char_p]),
     "hmg_set_stage_timing": (c_int, [c_int]),
     "hmg_stage_times": (c_int, [c_p]),
     "hmg_stage_counts": (c_int, [c_p]),
@@ -162,6 +166,12 @@ class Profile:
         """Gumbel (mu_msv, lambda, mu_vit, lambda) fitted on the GPU (hmg_calibrate)."""
         ev = hmg_evparams()
         _check(lib().hmg_calibrate(self._h, n, L, seed, lam, ctypes.byref(ev)), "hmg_calibrate")
+        return (ev.mu_msv, ev.lambda_msv, ev.mu_vit, ev.lambda_vit)
+
+    def calibrate_db(self, db, lam: float = 0.6931471805599453):
+        """Gumbel (mu_msv, lambda, mu_vit, lambda) fitted on the GPU scores of ``db`` (hmg_calibrate_db)."""
+        ev = hmg_evparams()
+        _check(lib().hmg_calibrate_db(self._h, db.handle, lam, ctypes.byref(ev)), "hmg_calibrate_db")
         return (ev.mu_msv, ev.lambda_msv, ev.mu_vit, ev.lambda_vit)
 
     def close(self):
@@ -362,7 +372,45 @@ def hmg_stage_counts() -> dict:
     return {"vit_pair_redo": int(c[0])}
 
 
+def hmg_prepare_thresholds(profile: Profile, F1: float = 0.02, F2: float = 1e-3, Lmax: int = 40000):
+    _check(lib().hmg_prepare_thresholds(profile.handle, F1, F2, Lmax), "hmg_prepare_thresholds")
+
+
+def set_tuning(name: str, value: int):
+    """Performance knob override (hmg_set_tuning); results never depend on it."""
+    _check(lib().hmg_set_tuning(name.encode(), int(value)), "hmg_set_tuning(%s)" % name)
+
+
+def clear_tuning(name: str | None = None):
+    _check(lib().hmg_clear_tuning(name.encode() if name else None), "hmg_clear_tuning")
+
+
+class tuning:
+    """with hmg.tuning(VIT_PAIR_W=4): ... -- overrides for the block, cleared after."""
+
+    def __init__(self, **kw):
+        self.kw = kw
+
+    def __enter__(self):
+        for k, v in self.kw.items():
+            set_tuning(k, v)
+        return self
+
+    def __exit__(self, *a):
+        for k in self.kw:
+            clear_tuning(k)
+
+
 # ------------------------------------------------------------------------ convenience
+def calibrated_profile(msc, tsc, device: int = 0, n: int = 1000, L: int = 200, seed: int = 7):
+    """A profile with its Gumbel locations fitted on the GPU (hmg_calibrate, lambda = ln 2,
+    P:41-45): profiles are immutable, so the searching profile is created with the fit."""
+    p = Profile(msc, tsc, device=device)
+    ev = p.calibrate(n=n, L=L, seed=seed)
+    p.close()
+    return Profile(msc, tsc, ev=ev, device=device), ev
+
+
 def alloc_outputs(nseq: int, device: int = 0):
     """Caller-owned device outputs for hmg_pipeline (torch provides the memory)."""
     import torch

@@ -158,9 +158,10 @@ class Database:
         np.cumsum(L, out=off[1:])
         total = int(off[-1])
         dsq = np.empty(total, dtype=np.uint8)
-        step = 1 << 24
+        step = 1 << 22
         shift = self.gstart[ids] - off[:-1]           # global position = local position + shift
-        for a in range(0, total, step):
+
+        def fill(a):
             b = min(total, a + step)
             j0 = int(np.searchsorted(off, a, side="right")) - 1
             j1 = int(np.searchsorted(off, b - 1, side="right"))
@@ -168,6 +169,16 @@ class Database:
             hi = np.minimum(off[j0 + 1:j1 + 1], b)
             pos = np.repeat(shift[j0:j1], hi - lo) + np.arange(a, b, dtype=np.int64)
             dsq[a:b] = _residues_at(self.seed, pos.astype(np.uint64))
+
+        chunks = range(0, total, step)
+        if len(chunks) > 1:                           # disjoint slices; numpy releases the GIL
+            import concurrent.futures as cf
+            import os
+            with cf.ThreadPoolExecutor(max_workers=min(len(chunks), os.cpu_count() or 1)) as ex:
+                list(ex.map(fill, chunks))
+        else:
+            for a in chunks:
+                fill(a)
         if len(self.planted_ids) and self.profile is not None:
             where = {int(s): j for j, s in enumerate(ids)}
             for s in self.planted_ids:

@@ -17,3 +17,15 @@ def pytest_configure(config):
 def cuda_available():
     import torch
     return torch.cuda.is_available()
+
+
+@pytest.fixture
+def tune():
+    """Set libhmg performance knobs (hmg_set_tuning) for one test; all cleared afterwards."""
+    from paper_conf_ipps_jiangg15_b200 import hmg
+    hmg.lib()
+
+    def set_(name, value):
+        hmg.set_tuning(name, int(value))
+    yield set_
+    hmg.clear_tuning()

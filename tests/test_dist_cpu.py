@@ -53,16 +53,19 @@ def _worker(rank, world, port, n, q):
     sv = torch.zeros(len(ids), dtype=torch.int32)
     sv[:len(local_surv)] = torch.as_tensor(local_surv)
     ns = torch.tensor([len(local_surv)], dtype=torch.int64)
-    words, gids, counts, surv = hdist.gather(hdist.pack_results(msv, vit, flags), sv, ns, torch.as_tensor(ids),
-                                             world)
+    words, gids, counts, surv = hdist.Gatherer(n, world, torch.as_tensor(ids))(msv, vit, flags, sv, ns)
+    g2 = hdist.Gatherer(n, world, torch.as_tensor(ids))
+    w2 = g2(msv, vit, flags, sv, ns)[0].clone()       # second step into the same static buffers
+    assert torch.equal(w2, words) and g2.nmax == max(hdist.shard_sizes(n, world))
     if rank == 0:
         q.put((words.numpy(), gids.numpy(), counts.numpy(), surv.numpy()))
     dist.barrier()
     dist.destroy_process_group()
 
 
-def test_gather_reassembles_global_order():
-    world, n = 2, 1001
+@pytest.mark.parametrize("world", [2, 3])
+def test_gather_reassembles_global_order(world):
+    n = 1001
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()

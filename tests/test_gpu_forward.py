@@ -233,11 +233,11 @@ def test_pipeline_forward_config3_full_size():
                                       (200, 12, 16), (200, 4, 16), (300, 1, 8), (300, 2, 8), (300, 4, 8), (300, 6, 8),
                                       (700, 1, 8), (700, 2, 8), (700, 3, 8), (300, 2, 16), (300, 4, 16),
                                       (300, 8, 16), (700, 1, 16), (700, 2, 16), (700, 4, 16)])
-def test_fwd_every_block_shape(M, S, qmax, monkeypatch):
+def test_fwd_every_block_shape(M, S, qmax, tune):
     """Every instantiated (W, Q, S): S sequences per block share the staged table and take
     sequences from the queue independently (named barriers per sequence group)."""
-    monkeypatch.setenv("HMG_FWD_S", str(S))
-    monkeypatch.setenv("HMG_FWD_QMAX", str(qmax))
+    tune("FWD_S", str(S))
+    tune("FWD_QMAX", str(qmax))
     rng = np.random.default_rng(M * 100 + S)
     prof = synth.make_profile(M, 9600 + M, dd=(1.0, 9.0))
     dsq, off = _ragged(rng, n=90, lmax=400)
@@ -248,10 +248,10 @@ def test_fwd_every_block_shape(M, S, qmax, monkeypatch):
 
 
 @pytest.mark.parametrize("M", [100, 257, 400, 512, 513, 1000, 2048, 3000])
-def test_fwd_lean_sixteen_nodes(M, monkeypatch):
-    """The register-lean 16-nodes-per-thread variant (HMG_FWD_QMAX=16: one warp up to M = 512, no
+def test_fwd_lean_sixteen_nodes(M, tune):
+    """The register-lean 16-nodes-per-thread variant (tuning FWD_QMAX=16: one warp up to M = 512, no
     per-row barrier; D = Dloc + c_in P applied as two 8-node product chains)."""
-    monkeypatch.setenv("HMG_FWD_QMAX", "16")
+    tune("FWD_QMAX", "16")
     rng = np.random.default_rng(M + 77)
     prof = synth.make_profile(M, 9700 + M, dd=(1.0, 9.0))
     dsq, off = _ragged(rng, n=50, lmax=400)

@@ -86,8 +86,8 @@ def test_msv_model_lengths(M):
 
 @pytest.mark.parametrize("G", [4, 8, 16, 32])
 @pytest.mark.parametrize("M", [60, 333, 900])
-def test_msv_every_lane_group(G, M, monkeypatch):
-    monkeypatch.setenv("HMG_MSV_G", str(G))
+def test_msv_every_lane_group(G, M, tune):
+    tune("MSV_G", str(G))
     rng = np.random.default_rng(G * 1000 + M)
     prof = synth.make_profile(M, M + G, stress=True)
     dsq, off = _ragged_db(rng, n=90, alphabet=29)
@@ -173,11 +173,11 @@ VMS = [1, 2, 3, 4, 5, 8, 9, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 
 @pytest.mark.parametrize("M", VMS)
 @pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
 @pytest.mark.parametrize("pair", [True, False])
-def test_vit_model_lengths(M, dd, pair, monkeypatch):
+def test_vit_model_lengths(M, dd, pair, tune):
     """pair: the s16x2 pair kernel (+ s32 re-scoring of what leaves its window); otherwise the
-    s32 kernels alone (HMG_NO_VIT_PAIR)."""
+    s32 kernels alone (tuning NO_VIT_PAIR)."""
     if not pair:
-        monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
+        tune("NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M + int(dd[0]))
     prof = synth.make_profile(M, 8000 + M, dd=dd)
     n = 40 if M <= 600 else 12
@@ -207,12 +207,12 @@ def test_vit_long_delete_chains(M):
 
 
 @pytest.mark.parametrize("pair", [True, False])
-def test_vit_long_delete_chains_s32(pair, monkeypatch):
+def test_vit_long_delete_chains_s32(pair, tune):
     """The delete-chain profiles above have -inf entry below node 1, so the pair kernel does not
     apply; here entry is finite everywhere but weak, so the pair kernel's Lazy-F (carries through
     both halves of every register, lane G-1 low -> lane 0 high) decides the score."""
     if not pair:
-        monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
+        tune("NO_VIT_PAIR", "1")
     for M in (3, 20, 64, 130, 300, 500, 700, 1000):
         rng = np.random.default_rng(M + 17)
         msc = np.full((M, 29), -6.0, np.float32)
@@ -235,8 +235,8 @@ def test_vit_long_delete_chains_s32(pair, monkeypatch):
 
 @pytest.mark.parametrize("G", [8, 16, 32])
 @pytest.mark.parametrize("M", [10, 100, 257, 600])
-def test_vit_pair_every_lane_group(G, M, monkeypatch):
-    monkeypatch.setenv("HMG_VIT_PAIR_G", str(G))
+def test_vit_pair_every_lane_group(G, M, tune):
+    tune("VIT_PAIR_G", str(G))
     rng = np.random.default_rng(G + M)
     prof = synth.make_profile(M, 300 + M + G, dd=(1.0, 9.0))
     dsq, off = _ragged_db(rng, n=70, alphabet=29, lmax=350)
@@ -332,6 +332,34 @@ def test_calibrate_matches_oracle_fit(M):
     assert p.calibrate(n=1000, L=200, seed=11) == (mu_m, lam_m, mu_v, lam_v)
 
 
+@pytest.mark.parametrize("M,lens", [(64, "fixed"), (400, "fixed"), (1500, "mixed")])
+def test_calibrate_db_equals_oracle_fit(M, lens):
+    """SURVEY 8(f) f3 parity: hmg_calibrate_db on a background DB vs the oracle's fit of the SAME
+    sequences (oracle raw scores -> nats -> bits with each sequence's null1 -> closed-form ML
+    location for lambda = ln 2).  The raw scores are bit-exact, so the two fits differ
+    only in the order of a double sum: 1e-9 relative."""
+    prof = synth.make_profile(M, 300 + M)
+    if lens == "fixed":
+        cal = synth.Database(np.full(1000, 200, np.int32), seed=7)
+    else:
+        cal = synth.make_db(1500, 5.4, 0.7, seed=19)
+    dsq, off = cal.materialize()
+    p = hmg.Profile(prof.msc, prof.tsc)
+    db = hmg.Database(dsq, off)
+    mu_m, lam_m, mu_v, lam_v = p.calibrate_db(db)
+    L = np.diff(off)
+    mraw = oracle.msv_db(oracle.MSVProfile(prof.msc), dsq, off)
+    vraw = oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)
+    mb = np.array([oracle.bits(oracle.msv_nats(int(r), int(l)), int(l)) for r, l in zip(mraw, L)])
+    vb = np.array([oracle.bits(oracle.vit_nats(int(r), int(l)), int(l)) for r, l in zip(vraw, L)])
+    lam = math.log(2)
+    want_m = oracle.fit_mu(mb[np.isfinite(mb)], lam)
+    want_v = oracle.fit_mu(vb[np.isfinite(vb)], lam)
+    assert lam_m == lam_v == pytest.approx(lam)
+    assert mu_m == pytest.approx(want_m, rel=1e-9, abs=1e-9)
+    assert mu_v == pytest.approx(want_v, rel=1e-9, abs=1e-9)
+
+
 def _check_pipeline(prof, dsq, off, F1, F2, sample=None):
     ev = _calibrate(prof)
     p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
@@ -408,11 +436,11 @@ def test_msv_config2_full_size_sampled():
 
 @pytest.mark.parametrize("M", [2, 3, 64, 255, 300, 513, 700, 1024, 1025, 1500, 2048, 2600, 4000])
 @pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
-def test_vit_block_kernel(M, dd, monkeypatch):
+def test_vit_block_kernel(M, dd, tune):
     """Block-per-sequence Viterbi (W warps per row, cross-warp Lazy-F through shared memory);
-    forced for small M with HMG_VIT_CTA, used by default above M = 512."""
-    monkeypatch.setenv("HMG_VIT_CTA", "1")
-    monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
+    forced for small M with tuning VIT_CTA, used by default above M = 512."""
+    tune("VIT_CTA", "1")
+    tune("NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M * 3 + int(dd[1]))
     prof = synth.make_profile(M, 9000 + M, dd=dd)
     n = 30 if M <= 1100 else 10
@@ -424,10 +452,10 @@ def test_vit_block_kernel(M, dd, monkeypatch):
 
 
 @pytest.mark.parametrize("M", [40, 300, 700, 2000])
-def test_vit_block_kernel_delete_chains(M, monkeypatch):
+def test_vit_block_kernel_delete_chains(M, tune):
     """D->D chains that cross every warp boundary of the block (cross-warp Lazy-F rounds)."""
-    monkeypatch.setenv("HMG_VIT_CTA", "1")
-    monkeypatch.setenv("HMG_NO_VIT_PAIR", "1")
+    tune("VIT_CTA", "1")
+    tune("NO_VIT_PAIR", "1")
     rng = np.random.default_rng(M + 5)
     msc = np.full((M, 29), -6.0, np.float32)
     msc[0, 0] = 4.0
@@ -449,16 +477,16 @@ def test_vit_block_kernel_delete_chains(M, monkeypatch):
                                                (1032, "2", 120, "s32"), (1032, "0", 300, "pair"),
                                                (60, "3", 300, "s32"), (1032, "0", 700, "pair"),
                                                (200, "2", 1000, "pair")])
-def test_pipeline_long_lane(chunk, sms, M, lane, monkeypatch):
+def test_pipeline_long_lane(chunk, sms, M, lane, tune):
     """The pipeline long lane: sequences longer than max(1500, 8 x mean) get chunked MSV (rows
     from the empty state M rows early) and whole-warp Viterbi on SMs held alone (the s32 latency
     lane, or the s16x2 pair lane for models of 129..1024 nodes).  Strong planted hits in some
     long sequences force the sequential fallback (a chunk sees a J->B row)."""
-    monkeypatch.setenv("HMG_PIPE_CHUNK", str(chunk))
+    tune("PIPE_CHUNK", str(chunk))
     if sms != "0":
-        monkeypatch.setenv("HMG_PIPE_LONG_SMS", sms)
+        tune("PIPE_LONG_SMS", sms)
     if lane == "s32":
-        monkeypatch.setenv("HMG_LONG_S32", "1")
+        tune("LONG_S32", "1")
     rng = np.random.default_rng(42)
     prof = synth.make_profile(M, 4242 + M)
     best = np.argmax(prof.msc[:, :20], axis=1).astype(np.uint8)
@@ -500,16 +528,17 @@ def test_pipeline_many_survivors(M):
 
 
 @pytest.mark.parametrize("M", [2, 3, 64, 300, 513, 1024, 1025, 1500, 2048, 2600, 4000])
-@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b"])
-def test_vit_block_pair_kernel(M, W, monkeypatch):
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t"])
+def test_vit_block_pair_kernel(M, W, tune):
     """Block-per-sequence pair kernel (W warps per row, 2 cells per register, closed-form carries
-    across virtual warps); forced for small M with HMG_VIT_PAIR_CTA, used by default above 1024.
-    W = 2 runs the kernel without a per-row barrier (vit_cpair2.cuh); "2b" the barrier kernel."""
-    monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
-    if W == "2b":
-        monkeypatch.setenv("HMG_VIT_CPAIR2_SG", "0")
+    across virtual warps); forced for small M with tuning VIT_PAIR_CTA, used by default above 1024.
+    W = 2 runs the kernel without a per-row barrier (vit_cpair2.cuh); "2b" the barrier kernel;
+    "2t" the barrier-free kernel with four transition vectors in shared memory (3 sequences/block)."""
+    tune("VIT_PAIR_CTA", "1")
+    if W in ("2b", "2t"):
+        tune("VIT_CPAIR2", "0" if W == "2b" else "23")
         W = 2
-    monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
+    tune("VIT_PAIR_W", str(W))
     rng = np.random.default_rng(M * 7 + W)
     for dd in [(7.0, 3.0), (1.0, 9.0)]:
         prof = synth.make_profile(M, 9100 + M + W, dd=dd)
@@ -521,15 +550,15 @@ def test_vit_block_pair_kernel(M, W, monkeypatch):
         assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)), dd
 
 
-@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b"])
-def test_vit_block_pair_delete_chains_and_exits(W, monkeypatch):
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t"])
+def test_vit_block_pair_delete_chains_and_exits(W, tune):
     """D->D chains across every virtual-warp boundary (low halves -> high halves), strong hits that
     re-base the window or overflow, and gap-only sequences handed to the s32 kernel."""
-    monkeypatch.setenv("HMG_VIT_PAIR_CTA", "1")
-    if W == "2b":
-        monkeypatch.setenv("HMG_VIT_CPAIR2_SG", "0")
+    tune("VIT_PAIR_CTA", "1")
+    if W in ("2b", "2t"):
+        tune("VIT_CPAIR2", "0" if W == "2b" else "23")
         W = 2
-    monkeypatch.setenv("HMG_VIT_PAIR_W", str(W))
+    tune("VIT_PAIR_W", str(W))
     for M in (40, 700, 2000):
         rng = np.random.default_rng(M + W)
         msc = np.full((M, 29), -6.0, np.float32)
@@ -554,11 +583,11 @@ def test_vit_block_pair_delete_chains_and_exits(W, monkeypatch):
 
 
 @pytest.mark.parametrize("M", [129, 300, 700, 1000])
-def test_vit_pair_maxplus_scan(M, monkeypatch):
+def test_vit_pair_maxplus_scan(M, tune):
     """the cross-lane D->D carries of the pair kernel resolved by one max-plus
-    prefix scan (HMG_VIT_SCAN) instead of vote-terminated passes: identical raw scores on the
+    prefix scan (tuning VIT_SCAN) instead of vote-terminated passes: identical raw scores on the
     typical and the long-D-chain (Dir(1, 9)) profiles and on chains crossing every lane."""
-    monkeypatch.setenv("HMG_VIT_SCAN", "1")
+    tune("VIT_SCAN", "1")
     rng = np.random.default_rng(M + 31)
     for dd in [(7.0, 3.0), (1.0, 9.0)]:
         prof = synth.make_profile(M, 600 + M, dd=dd)
@@ -582,18 +611,16 @@ def test_vit_pair_maxplus_scan(M, monkeypatch):
     assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(msc, tsc), dsq, off))
 
 
-@pytest.mark.parametrize("cfg,sched", [(1, None), (3, None), (3, (12, 700, 1)), (3, (2, 1500, 1)),
-                                       (3, (6, 1000, 0)), (1, (12, 1000, 0))])
-def test_pipeline_upload_overlapped_equals_pipeline(cfg, sched, monkeypatch):
+@pytest.mark.parametrize("cfg,sched", [(1, None), (3, None), (3, (12, 700)), (3, (2, 1500)),
+                                       (3, (6, 1000)), (1, (12, 1000))])
+def test_pipeline_upload_overlapped_equals_pipeline(cfg, sched, tune):
     """hmg_pipeline_upload (packed image re-sent from pinned host memory in length-ordered parts,
     MSV per part as it lands, long lane alongside) gives hmg_pipeline's outputs exactly; the device
     image is scrubbed first so every residue read must come from this call's upload.  `sched`
-    overrides the part schedule (HMG_UPLOAD_PARTS, HMG_UPLOAD_GROW: shrinking / growing parts;
-    HMG_UPLOAD_GATED: one MSV launch waiting on per-part landing flags, or one launch per part)."""
+    overrides the part schedule (tuning UPLOAD_PARTS, UPLOAD_GROW: shrinking / growing parts)."""
     if sched is not None:
-        monkeypatch.setenv("HMG_UPLOAD_PARTS", str(sched[0]))
-        monkeypatch.setenv("HMG_UPLOAD_GROW", str(sched[1]))
-        monkeypatch.setenv("HMG_UPLOAD_GATED", str(sched[2]))
+        tune("UPLOAD_PARTS", sched[0])
+        tune("UPLOAD_GROW", sched[1])
     prof, db = synth.config(cfg)
     dsq, off = db.materialize()
     ev = _calibrate(prof) if cfg == 1 else (-9.5, math.log(2), -9.0, math.log(2))
@@ -651,3 +678,40 @@ def test_pipeline_in_cuda_graph():
         sv = ref["survivor_ids"][:ns].long()
         assert torch.equal(out["survivor_ids"][:ns], ref["survivor_ids"][:ns])
         assert torch.equal(out["vit_raw"][sv], ref["vit_raw"][sv])
+
+
+def test_graph_survives_new_thresholds():
+    """Threshold tables are never freed while the profile lives: a graph captured with
+    one (F1, F2) still replays its outputs after eager calls built tables for other F; a fresh
+    profile prepared with hmg_prepare_thresholds captures on its first call."""
+    prof, db = synth.config(1)
+    dsq, off = db.materialize()
+    ev = _calibrate(prof)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    D = hmg.Database(dsq, off)
+    ref = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline(p, D, F1=0.2, F2=0.1, **ref)
+    out = hmg.alloc_outputs(D.nseq)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, capture_error_mode="thread_local"):
+        hmg.hmg_pipeline(p, D, F1=0.2, F2=0.1, stream=torch.cuda.current_stream(), **out)
+    other = hmg.alloc_outputs(D.nseq)
+    for F1, F2 in ((0.05, 0.01), (0.5, 0.5), (0.9, 0.02)):          # new tables (a larger set each)
+        hmg.hmg_pipeline(p, D, F1=F1, F2=F2, **other)
+    g.replay()
+    torch.cuda.synchronize()
+    for k in ("msv_raw", "flags", "n_survivors"):
+        assert torch.equal(out[k], ref[k]), k
+    assert int(other["n_survivors"].item()) != int(ref["n_survivors"].item())
+    # first call under capture: tables prepared ahead
+    p2 = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    hmg.hmg_prepare_thresholds(p2, 0.2, 0.1, Lmax=int(np.diff(off).max()))
+    out2 = hmg.alloc_outputs(D.nseq)
+    g2 = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g2, capture_error_mode="thread_local"):
+        hmg.hmg_pipeline(p2, D, F1=0.2, F2=0.1, stream=torch.cuda.current_stream(), **out2)
+    g2.replay()
+    torch.cuda.synchronize()
+    for k in ("msv_raw", "flags", "n_survivors"):
+        assert torch.equal(out2[k], ref[k]), k
+

@@ -179,3 +179,19 @@ def test_forward_geometry_host_only(L):
         assert (q["fwd_lanes"], q["fwd_nodes"], q["fwd_warps"]) == (T, Qn, max(1, T // 32)), M
     p = hmg.Profile(np.zeros((4097, 29), np.float32), np.full((4097, 8), -1.0, np.float32), device=-1)
     assert p.quant()["fwd_warps"] == 0
+
+
+def test_tuning_api():
+    """hmg_set_tuning accepts the documented knobs only (the library reads no environment
+    variables); clearing restores the defaults."""
+    hmg.lib()
+    for k in ("MSV_G", "VIT_PAIR_W", "VIT_CPAIR2", "UPLOAD_PARTS", "PIPE_LLONG"):
+        hmg.set_tuning(k, 4)
+        hmg.clear_tuning(k)
+    with pytest.raises(hmg.HmgError):
+        hmg.set_tuning("NOT_A_KNOB", 1)
+    with pytest.raises(hmg.HmgError):
+        hmg.clear_tuning("NOT_A_KNOB")
+    hmg.clear_tuning()
+    src = open(os.path.join(os.path.dirname(__file__), "..", "paper_conf_ipps_jiangg15_b200", "csrc", "host.cu")).read()
+    assert "getenv" not in src

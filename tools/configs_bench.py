@@ -59,8 +59,7 @@ def report(cfg, M, D, ms, st, extra):
 
 
 def pipeline(cfg, prof, dsq, off):
-    ev = hdist.calibrate(prof.msc, prof.tsc)
-    P = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    P, ev = hmg.calibrated_profile(prof.msc, prof.tsc)
     D = hmg.Database(dsq, off)
     out = hmg.alloc_outputs(D.nseq)
     ms, st = timed(lambda: hmg.hmg_pipeline(P, D, **out))

@@ -1,5 +1,5 @@
 """Forward stage on the Viterbi passes of BASELINE config 3 (the bench's Forward leg): lengths of
-the Forward list and the stage time per geometry (HMG_FWD_W / HMG_FWD_S overrides).
+the Forward list and the stage time per geometry (tuning FWD_W / FWD_S).
 usage: python tools/fwd_latency.py"""
 import os, sys, json, subprocess
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -10,9 +10,8 @@ from paper_conf_ipps_jiangg15_b200 import build, hmg, synth, dist as hdist
 build.build()
 prof, db = synth.config(3)
 dsq, off = db.materialize()
-ev = hdist.calibrate(prof.msc, prof.tsc)
 D = hmg.Database(dsq, off)
-P = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+P, ev = hmg.calibrated_profile(prof.msc, prof.tsc)
 out = hmg.alloc_outputs(D.nseq)
 fo = hmg.alloc_forward_outputs(D.nseq)
 hmg.hmg_pipeline_forward(P, D, **out, **fo)
@@ -24,7 +23,7 @@ print(json.dumps({"n_fwd": nf, "residues": int(L.sum()), "top_lengths": sorted(L
 res = torch.zeros(D.nseq, dtype=torch.float32, device="cuda")
 hmg.hmg_set_stage_timing(True)
 for W in (1, 2, 4, 8, 16):
-    os.environ["HMG_FWD_W"] = str(W)
+    hmg.set_tuning("FWD_W", W)
     try:
         Pw = hmg.Profile(prof.msc, prof.tsc)
     except hmg.HmgError:

@@ -13,7 +13,7 @@ Ms = [int(m) for m in sys.argv[1].split(",")] if len(sys.argv) > 1 else [64, 100
 for M in Ms:
     prof = synth.make_profile(M, 1000 + M)
     for G in (4, 8, 16, 32):
-        os.environ["HMG_MSV_G"] = str(G)
+        hmg.set_tuning("MSV_G", G)
         P = hmg.Profile(prof.msc)
         q = P.quant()
         if q["msv_lanes"] != G:

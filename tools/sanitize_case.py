@@ -10,8 +10,10 @@ rng = np.random.default_rng(0)
 lens = [int(x) for x in rng.integers(5, 300, size=120)] + [1700, 2100]   # two long-lane sequences
 dsq = np.concatenate([synth.random_dsq(rng, L, 29) for L in lens]).astype(np.uint8)
 off = np.zeros(len(lens) + 1, np.int64); np.cumsum(lens, out=off[1:])
-for M, env in ((60, {}), (300, {}), (700, {}), (3500, {}), (90, {"HMG_VIT_CTA": "1"})):
-    os.environ.update(env)
+for M, env in ((60, {}), (300, {}), (700, {}), (1500, {}), (2048, {"VIT_CPAIR2": 23}), (3500, {}),
+               (90, {"VIT_CTA": 1})):
+    for k, v in env.items():
+        hmg.set_tuning(k, v)
     prof = synth.make_profile(M, M, dd=(1.0, 9.0))
     P = hmg.Profile(prof.msc, prof.tsc, ev=(-9.0, 0.693, -9.0, 0.693))
     D = hmg.Database(dsq, off)
@@ -22,8 +24,7 @@ for M, env in ((60, {}), (300, {}), (700, {}), (3500, {}), (90, {"HMG_VIT_CTA": 
     vr = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
     hmg.hmg_viterbi(P, D, vr)
     torch.cuda.synchronize()
-    for k in env:
-        del os.environ[k]
+    hmg.clear_tuning()
     print("M", M, "ok", int(out["n_survivors"].item()))
 msc = np.full((40, 29), 30.0, np.float32)       # exact MSV kernel (bias >= 66 + tbm)
 P = hmg.Profile(msc)

@@ -11,8 +11,7 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 build.build()
 prof, db = synth.config(cfg)
 t = time.time(); dsq, off = db.materialize(); tm = time.time() - t
-ev = hdist.calibrate(prof.msc, prof.tsc)
-P = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+P, ev = hmg.calibrated_profile(prof.msc, prof.tsc)
 t = time.time(); D = hmg.Database(dsq, off); tp = time.time() - t
 out = hmg.alloc_outputs(D.nseq)
 M = prof.M

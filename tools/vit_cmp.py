@@ -18,9 +18,9 @@ for M in Ms:
     outs = {}
     for mode in ("pair", "s32"):
         if mode == "s32":
-            os.environ["HMG_NO_VIT_PAIR"] = "1"
+            hmg.set_tuning("NO_VIT_PAIR", 1)
         P = hmg.Profile(prof.msc, prof.tsc)
-        os.environ.pop("HMG_NO_VIT_PAIR", None)
+        hmg.clear_tuning("NO_VIT_PAIR")
         q = P.quant()
         raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
         best = None

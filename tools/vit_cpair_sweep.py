@@ -14,14 +14,14 @@ prof = synth.make_profile(M, 1000 + M)
 hmg.hmg_set_stage_timing(True)
 ref = None
 for mode in ("s32", "W2S2", "W2S4", "W4S1", "W4S3", "W8S1", "W8S2"):
-    for k in ("HMG_NO_VIT_PAIR", "HMG_VIT_PAIR_W", "HMG_VIT_PAIR_SG"):
-        os.environ.pop(k, None)
+    for k in ("NO_VIT_PAIR", "VIT_PAIR_W", "VIT_PAIR_SG", "VIT_CPAIR2"):
+        hmg.clear_tuning(k)
     if mode == "s32":
-        os.environ["HMG_NO_VIT_PAIR"] = "1"
+        hmg.set_tuning("NO_VIT_PAIR", 1)
     else:
         w, sg = mode[1:].split("S")
-        os.environ["HMG_VIT_PAIR_W"] = w
-        os.environ["HMG_VIT_PAIR_SG"] = sg
+        hmg.set_tuning("VIT_PAIR_W", int(w))
+        hmg.set_tuning("VIT_PAIR_SG", int(sg))
     P = hmg.Profile(prof.msc, prof.tsc)
     q = P.quant()
     raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")

@@ -17,9 +17,9 @@ for M in (200, 400, 700, 1000):
         outs = []
         for mode in ("passes", "scan"):
             if mode == "scan":
-                os.environ["HMG_VIT_SCAN"] = "1"
+                hmg.set_tuning("VIT_SCAN", 1)
             P = hmg.Profile(prof.msc, prof.tsc)
-            os.environ.pop("HMG_VIT_SCAN", None)
+            hmg.clear_tuning("VIT_SCAN")
             raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
             best = None
             for _ in range(3):

@@ -7,8 +7,7 @@ from paper_conf_ipps_jiangg15_b200 import build, hmg, synth, dist as hdist
 build.build()
 prof, db = synth.config(3)
 dsq, off = db.materialize()
-ev = hdist.calibrate(prof.msc, prof.tsc)
-P = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+P, ev = hmg.calibrated_profile(prof.msc, prof.tsc)
 D = hmg.Database(dsq, off)
 out = hmg.alloc_outputs(D.nseq)
 hmg.hmg_pipeline(P, D, **out)

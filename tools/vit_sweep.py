@@ -15,7 +15,7 @@ for M in Ms:
     prof = synth.make_profile(M, 1000 + M)
     ref = None
     for G in (8, 16, 32):
-        os.environ["HMG_VIT_PAIR_G"] = str(G)
+        hmg.set_tuning("VIT_PAIR_G", G)
         P = hmg.Profile(prof.msc, prof.tsc)
         q = P.quant()
         raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
