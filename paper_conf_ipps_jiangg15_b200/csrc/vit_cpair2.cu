@@ -22,6 +22,7 @@ const void* pick2(int q, size_t* smem) {
 const void* cpair2_ptr(int var, int Q, size_t* smem) {
   switch (var) {
     case 2: return pick2<2, 0, 2, 16>(Q, smem);
+    case 12: return pick2<2, 1, 8, 16>(Q, smem);
     case 22: return pick2<2, 2, 2, 16>(Q, smem);
     case 23: return pick2<3, 2, 8, 16>(Q, smem);
   }

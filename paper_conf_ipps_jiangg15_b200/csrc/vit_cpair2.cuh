@@ -31,7 +31,8 @@
 // -- is vit_pair.cuh's.
 //
 // Registers set the sequences in flight (two warps of 64 K 32-bit registers per SM).  TSM = 0 keeps
-// all seven transition vectors in registers (255 registers: 4 sequences per SM); TSM = 2 streams
+// all seven transition vectors in registers (255 registers: 4 sequences per SM); TSM = 1 streams
+// the two only the I update uses (tMI, tII) from shared memory; TSM = 2 streams
 // the four that phase A uses (tMM, tIM, tMI, tII) from shared memory, one copy per block (about
 // 160 registers: 6 sequences per SM at the cost of 8 more bytes of shared-memory reads per cell).
 #pragma once
@@ -77,6 +78,23 @@ __device__ __forceinline__ void store_row(uint32_t* row, int z, const uint32_t (
   if constexpr (C::has2)
     *reinterpret_cast<uint2*>(row + C::n4 * 4 * G + z * 2) = make_uint2(v[4 * C::n4], v[4 * C::n4 + 1]);
   if constexpr (C::has1) row[(C::n4 * 4 + (C::has2 ? 2 : 0)) * G + z] = v[Q - 1];
+}
+
+// load_row from a 32-bit shared-memory address (ld.shared: no generic-to-shared conversion per row)
+template <int G, int Q>
+__device__ __forceinline__ void lds_row(uint32_t row_s, int z, uint32_t (&e)[Q]) {
+  using C = Chunks<Q>;
+#pragma unroll
+  for (int c = 0; c < C::n4; ++c)
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(e[4 * c]), "=r"(e[4 * c + 1]), "=r"(e[4 * c + 2]), "=r"(e[4 * c + 3])
+                 : "r"(row_s + (uint32_t)(c * 4 * G + z * 4) * 4u));
+  if constexpr (C::has2)
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(e[4 * C::n4]), "=r"(e[4 * C::n4 + 1])
+                 : "r"(row_s + (uint32_t)(C::n4 * 4 * G + z * 2) * 4u));
+  if constexpr (C::has1)
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(e[Q - 1])
+                 : "r"(row_s + (uint32_t)((C::n4 * 4 + (C::has2 ? 2 : 0)) * G + z) * 4u));
 }
 
 // s16x2 with both halves clamped below at -32768 (tDD sums: relu(c + sum) is exact with the clamp)
@@ -125,16 +143,15 @@ __global__ void __launch_bounds__(64 * SG, (TSM && SG == 3) ? 2 : 1) vit_cpair2_
   const int bmine = bfull + 1 + 2 * w;           // + parity: this warp published a row
   const int bother = bfull + 3 - 2 * w;          // + parity: the other warp published a row
 
-  constexpr int QR = TSM ? 1 : Q;                // register copies of tMM, tIM, tMI, tII
-  uint32_t tMM[QR], tIM[QR], tMI[QR], tII[QR];
+  constexpr int QR = TSM == 2 ? 1 : Q;           // register copies of tMM, tIM (TSM 2: shared memory)
+  constexpr int QI = TSM ? 1 : Q;                // register copies of tMI, tII (TSM 1, 2: shared memory)
+  uint32_t tMM[QR], tIM[QR], tMI[QI], tII[QI];
   uint32_t tDM[Q], tMD[Q], tDD[Q];
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
     const int o = g * Q + q;
-    if constexpr (!TSM) {
-      tMM[q] = tr[1 * NT * Q + o]; tIM[q] = tr[2 * NT * Q + o]; tMI[q] = tr[5 * NT * Q + o];
-      tII[q] = tr[6 * NT * Q + o];
-    }
+    if constexpr (TSM < 2) { tMM[q] = tr[1 * NT * Q + o]; tIM[q] = tr[2 * NT * Q + o]; }
+    if constexpr (TSM == 0) { tMI[q] = tr[5 * NT * Q + o]; tII[q] = tr[6 * NT * Q + o]; }
     tDM[q] = tr[3 * NT * Q + o]; tMD[q] = tr[4 * NT * Q + o]; tDD[q] = tr[7 * NT * Q + o];
   }
   // per half: sum of the thread's tDD (bs), prefix up to its last node (s31), warp-exclusive prefix (pbs)
@@ -174,6 +191,7 @@ __global__ void __launch_bounds__(64 * SG, (TSM && SG == 3) ? 2 : 1) vit_cpair2_
   const long long ntot = a.list ? *a.nlist : a.nseq;
   const int safe = a.safe;
   const uint32_t* rare = reinterpret_cast<const uint32_t*>(a.rsc);
+  const uint32_t tab_s = (uint32_t)__cvta_generic_to_shared(sm);      // emission rows (shared window)
 
   for (;;) {
     if (g == 0) *s_next = (long long)atomicAdd(a.counter, 1ull);
@@ -245,24 +263,33 @@ __global__ void __launch_bounds__(64 * SG, (TSM && SG == 3) ? 2 : 1) vit_cpair2_
             else { q0 = Q - 1; nq = 1; off = (C::n4 * 4 + (C::has2 ? 2 : 0)) * NT + g; }
             uint32_t tmm[4], tim[4], tmi[4], tii[4];
             if (nq == 4) {
-              const uint4 v0 = *reinterpret_cast<const uint4*>(ttab + 0 * ROWW + off);
-              const uint4 v1 = *reinterpret_cast<const uint4*>(ttab + 1 * ROWW + off);
+              if constexpr (TSM == 2) {
+                const uint4 v0 = *reinterpret_cast<const uint4*>(ttab + 0 * ROWW + off);
+                const uint4 v1 = *reinterpret_cast<const uint4*>(ttab + 1 * ROWW + off);
+                tmm[0] = v0.x; tmm[1] = v0.y; tmm[2] = v0.z; tmm[3] = v0.w;
+                tim[0] = v1.x; tim[1] = v1.y; tim[2] = v1.z; tim[3] = v1.w;
+              }
               const uint4 v2 = *reinterpret_cast<const uint4*>(ttab + 2 * ROWW + off);
               const uint4 v3 = *reinterpret_cast<const uint4*>(ttab + 3 * ROWW + off);
-              tmm[0] = v0.x; tmm[1] = v0.y; tmm[2] = v0.z; tmm[3] = v0.w;
-              tim[0] = v1.x; tim[1] = v1.y; tim[2] = v1.z; tim[3] = v1.w;
               tmi[0] = v2.x; tmi[1] = v2.y; tmi[2] = v2.z; tmi[3] = v2.w;
               tii[0] = v3.x; tii[1] = v3.y; tii[2] = v3.z; tii[3] = v3.w;
             } else if (nq == 2) {
-              const uint2 v0 = *reinterpret_cast<const uint2*>(ttab + 0 * ROWW + off);
-              const uint2 v1 = *reinterpret_cast<const uint2*>(ttab + 1 * ROWW + off);
+              if constexpr (TSM == 2) {
+                const uint2 v0 = *reinterpret_cast<const uint2*>(ttab + 0 * ROWW + off);
+                const uint2 v1 = *reinterpret_cast<const uint2*>(ttab + 1 * ROWW + off);
+                tmm[0] = v0.x; tmm[1] = v0.y; tim[0] = v1.x; tim[1] = v1.y;
+              }
               const uint2 v2 = *reinterpret_cast<const uint2*>(ttab + 2 * ROWW + off);
               const uint2 v3 = *reinterpret_cast<const uint2*>(ttab + 3 * ROWW + off);
-              tmm[0] = v0.x; tmm[1] = v0.y; tim[0] = v1.x; tim[1] = v1.y;
               tmi[0] = v2.x; tmi[1] = v2.y; tii[0] = v3.x; tii[1] = v3.y;
             } else {
-              tmm[0] = ttab[0 * ROWW + off]; tim[0] = ttab[1 * ROWW + off];
+              if constexpr (TSM == 2) { tmm[0] = ttab[0 * ROWW + off]; tim[0] = ttab[1 * ROWW + off]; }
               tmi[0] = ttab[2 * ROWW + off]; tii[0] = ttab[3 * ROWW + off];
+            }
+            if constexpr (TSM == 1) {
+#pragma unroll
+              for (int jj = 0; jj < 4; ++jj)
+                if (jj < nq) { tmm[jj] = tMM[q0 + jj]; tim[jj] = tIM[q0 + jj]; }
             }
 #pragma unroll
             for (int j = nq - 1; j >= 0; --j) {
@@ -415,10 +442,10 @@ __global__ void __launch_bounds__(64 * SG, (TSM && SG == 3) ? 2 : 1) vit_cpair2_
       // ---------------- phase B: M(i, .) (Alg 2 l.16 + emission, reading R15), row max, D chain
       {
         uint32_t e[Q];
-        if (x < 20 || x == 26) {
-          load_row<NT, Q>(sm + (x < 20 ? x : 20) * ROWW, g, e);     // shared memory
-        } else {
-          load_row<NT, Q>(rare + x * ROWW, g, e);                    // rare codes: L2
+        if (x < 20 || x == 26) {                  // shared memory
+          lds_row<NT, Q>(tab_s + (uint32_t)((x < 20 ? x : 20) * ROWW) * 4u, g, e);
+        } else {                                   // rare codes (B J Z O U, gaps): L2
+          load_row<NT, Q>(rare + x * ROWW, g, e);
         }
 #pragma unroll
         for (int q = Q - 1; q >= 0; --q) {

@@ -434,6 +434,84 @@ def test_msv_config2_full_size_sampled():
     assert np.array_equal(got[sample], want)
 
 
+def _stratified(lengths, n, rng):
+    """n sequence ids spread over the length distribution (equal counts per length decile)."""
+    order = np.argsort(lengths, kind="stable")
+    parts = np.array_split(order, 10)
+    return np.unique(np.concatenate([rng.choice(pp, n // 10, replace=False) for pp in parts]))
+
+
+def test_viterbi_config4_full_size_sampled():
+    """BASELINE config 4 at full size in the bench launch configuration: the Viterbi filter
+    (Lazy-F) over every one of the 550k Swiss-Prot-shaped sequences at M = 2048 (the two-warp
+    kernel, M up to 2405 P:816-818).  The oracle checks a 2k length-stratified sample,
+    the 50 longest sequences (L up to 35,213) and the pass flags there; planted homologs (strong
+    hits that re-base the 16-bit window) are checked on a second 20k-sequence DB."""
+    c = synth.CONFIGS[4]
+    prof = synth.make_profile(c["M"], c["pseed"])
+    db = synth.make_db(c["N"], c["mu_ln"], c["sigma"], c["dseed"])
+    dsq, off = db.materialize()
+    ev = _calibrate(prof)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    assert p.quant()["vit_pair_lanes"] == 64                       # the two-warp pair kernel
+    D = hmg.Database(dsq, off)
+    raw = torch.full((D.nseq,), -12345, dtype=torch.int16, device="cuda")
+    pas = torch.zeros(D.nseq, dtype=torch.uint8, device="cuda")
+    hmg.hmg_viterbi(p, D, raw, pass_=pas, F2=1e-3)
+    torch.cuda.synchronize()
+    got = raw.cpu().numpy().astype(np.int32)
+    gp = pas.cpu().numpy()
+    assert (got != -12345).all()
+    rng = np.random.default_rng(4)
+    sample = np.unique(np.concatenate([_stratified(db.lengths, 2000, rng), np.argsort(-db.lengths)[:50]]))
+    assert db.lengths[sample].max() > 30000
+    vp = oracle.VitProfile(prof.msc, prof.tsc)
+    want = oracle.vit_db(vp, dsq, off, ids=sample)
+    assert np.array_equal(got[sample], want)
+    wp = [oracle.vit_pass(int(r), int(db.lengths[s]), ev[2], ev[3], 1e-3) for r, s in zip(want, sample)]
+    assert np.array_equal(gp[sample], np.array(wp, np.uint8))
+    # planted homologs: strong hits
+    db2 = synth.make_db(20000, c["mu_ln"], c["sigma"], 44, planted=0.01, profile=prof)
+    dsq2, off2 = db2.materialize()
+    D2 = hmg.Database(dsq2, off2)
+    raw2 = torch.zeros(D2.nseq, dtype=torch.int16, device="cuda")
+    hmg.hmg_viterbi(p, D2, raw2)
+    torch.cuda.synchronize()
+    ids = np.unique(np.concatenate([db2.planted_ids, rng.choice(db2.N, 300, replace=False)]))
+    w2 = oracle.vit_db(vp, dsq2, off2, ids=ids)
+    assert np.array_equal(raw2.cpu().numpy().astype(np.int32)[ids], w2)
+    assert (w2[np.isin(ids, db2.planted_ids)] > 10000).mean() > 0.5     # they are hits
+
+
+@pytest.mark.parametrize("which", [0, 1, 2])
+def test_pipeline_config5_shard_full_size_sampled(which):
+    """BASELINE config 5 as one rank of the 8-way run holds it: the 1/8 snake shard (1.25 M
+    sequences) of the 10 M-sequence UniProt-shaped DB at M = 100 / 500 / 1000, the pipeline in the
+    bench launch configuration; the oracle checks a 3k length-stratified sample, the 40 longest and
+    every survivor among them (_check_pipeline) plus 2000 random survivors' Viterbi scores."""
+    from paper_conf_ipps_jiangg15_b200 import dist as hdist
+    c = synth.CONFIGS[5]
+    prof = synth.make_profile(c["M"][which], c["pseed"][which])
+    db = synth.make_db(c["N"], c["mu_ln"], c["sigma"], c["dseed"])
+    ids = hdist.snake_shard(db.lengths, 8, 0)
+    dsq, off = db.materialize(ids)
+    L = np.diff(off)
+    rng = np.random.default_rng(50 + which)
+    sample = np.unique(np.concatenate([_stratified(L, 3000, rng), np.argsort(-L)[:40]]))
+    _check_pipeline(prof, dsq, off, F1=0.02, F2=1e-3, sample=sample)
+    ev = _calibrate(prof)
+    p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
+    D = hmg.Database(dsq, off)
+    out = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline(p, D, F1=0.02, F2=1e-3, **out)
+    torch.cuda.synchronize()
+    ns = int(out["n_survivors"].item())
+    surv = out["survivor_ids"].cpu().numpy()[:ns]
+    pick = rng.choice(surv, min(2000, ns), replace=False)
+    want = oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off, ids=pick)
+    assert np.array_equal(out["vit_raw"].cpu().numpy().astype(np.int32)[pick], want)
+
+
 @pytest.mark.parametrize("M", [2, 3, 64, 255, 300, 513, 700, 1024, 1025, 1500, 2048, 2600, 4000])
 @pytest.mark.parametrize("dd", [(7.0, 3.0), (1.0, 9.0)])
 def test_vit_block_kernel(M, dd, tune):

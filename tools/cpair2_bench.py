@@ -14,7 +14,7 @@ D = hmg.Database(dsq, off)
 prof = synth.make_profile(M, 1000 + M)
 hmg.hmg_set_stage_timing(True)
 ref = None
-for sg in ("0", "2", "22", "23"):
+for sg in ("0", "2", "12", "22", "23"):
     hmg.set_tuning("VIT_CPAIR2", int(sg))
     P = hmg.Profile(prof.msc, prof.tsc)
     raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")

@@ -1,7 +1,8 @@
 """Executed SASS opcode mix per DP cell from an ncu report with source counters (the
 `--set full --import-source on` captures of tools/gpu_run.sh): lane-instructions per cell by
 opcode, i.e. the measured counterpart of the per-cell operation counts in DESIGN.md.
-usage: python tools/sass_mix.py report.ncu-rep cells [top]"""
+usage: python tools/sass_mix.py report.ncu-rep|source.csv cells [top]
+(source.csv: `ncu -i report --page source --csv --print-source sass` output)"""
 import collections
 import csv
 import io
@@ -10,8 +11,11 @@ import sys
 
 rep, cells = sys.argv[1], float(sys.argv[2])
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 20
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                     capture_output=True, text=True).stdout
+if rep.endswith(".csv"):
+    out = open(rep).read()
+else:
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                         capture_output=True, text=True).stdout
 lines = out.splitlines()
 kname = lines[0].split(",", 1)[1].strip().strip('"') if lines else "?"
 rows = list(csv.reader(io.StringIO("\n".join(lines[1:]))))
