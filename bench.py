@@ -315,7 +315,7 @@ def configs_leg(args, dev, stream, flush, p_int, ev_file):
                 raw = torch.empty(n, dtype=torch.uint8, device=dev)
                 pas = torch.empty(n, dtype=torch.uint8, device=dev)
                 fn = lambda: hmg.hmg_msv(P, D2, raw, pas, F1=args.F1, stream=stream)
-                key, ops, stage = "msv_fast_kernel", MSV_ALU_OPS_PER_CELL, "msv_kernel"
+                key, ops, stage = "msv_fast_kernel<8,13>", MSV_ALU_OPS_PER_CELL, "msv_kernel"   # no mix: ALU only
             else:
                 raw = torch.empty(n, dtype=torch.int16, device=dev)
                 pas = torch.empty(n, dtype=torch.uint8, device=dev)
@@ -557,7 +557,9 @@ def main():
         roofline["survey_8d_msv_ratio"] = round(msv_gcups * 1e9 / (p_int * 1e12 / 2), 3) if msv_gcups else None
     roofline["peak_source"] = "%s sm_max_mhz x %d SMs x %d lanes/clk (ALU pipe, measured profiles/intpeak_r01.txt)" \
                               % (src, nsm, ALU_LANES_PER_CLK_SM)
-    tb, tsrc = load_traffic("msv_fast_kernel") if args.stage != "vit" else (None, None)
+    ek = evf.get("vit_cpair2_kernel" if args.stage == "vit" and q["vit_pair_lanes"] == 64 else
+                  "msv_fast_kernel" if args.stage != "vit" else "-", {})
+    tb, tsrc = ek.get("dram_bytes_per_launch"), ek.get("dram_source")
     roofline["traffic"] = tb
     roofline["traffic_unit"] = "bytes/launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
     roofline["traffic_source"] = tsrc
