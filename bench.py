@@ -387,6 +387,9 @@ def main():
     ap.add_argument("--batch", type=int, default=64, help="profiles of the f4 batch leg (0 = skip)")
     ap.add_argument("--cpu-sample-every", type=int, default=0, help="default: 2 (pipeline, msv), 23 (vit)")
     ap.add_argument("--ref-sample", type=int, default=100000)
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo + --one-device: exercise the N > 1 path with every rank on cuda:0 (tests only)")
+    ap.add_argument("--one-device", action="store_true", help="every rank on cuda:0 (tests of the N > 1 path)")
     ap.add_argument("--tune", action="append", default=[], metavar="NAME=V",
                     help="libhmg performance knob (hmg_set_tuning; sweeps only, results never depend on it)")
     args = ap.parse_args()
@@ -397,6 +400,8 @@ def main():
         args.cpu_sample_every = 23 if args.stage == "vit" else 2   # ~10 s of oracle work on 16 cores
 
     rank, world, local = env_rank()
+    if args.one_device:
+        local = 0
     if args.gpus != world and not (args.impl == "reference" and world == 1):
         sys.exit("bench.py: --gpus %d but WORLD_SIZE %d (launch N > 1 with torchrun, one process per GPU)"
                  % (args.gpus, world))
@@ -411,7 +416,10 @@ def main():
     from paper_conf_ipps_jiangg15_b200 import dist as hdist
 
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if rank == 0:
@@ -437,7 +445,7 @@ def main():
     out = hmg.alloc_outputs(n, local)
     vraw = torch.zeros(n, dtype=torch.int16, device=dev) if args.stage == "vit" else out["vit_raw"]
     gids = torch.as_tensor(ids, device=dev)
-    gather = hdist.Gatherer(gdb.N, world, gids) if world > 1 else None
+    gather = hdist.Gatherer(gdb.N, world, gids, stage_host=args.backend == "gloo") if world > 1 else None
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
@@ -511,7 +519,8 @@ def main():
     torch.cuda.synchronize()
     ms = [a.elapsed_time(b) for a, b in evs]
     t_step = sum(ms) / len(ms)
-    t_max = torch.tensor([t_step], dtype=torch.float64, device=dev)
+    rdev = dev if args.backend == "nccl" else torch.device("cpu")        # gloo tests: host reductions
+    t_max = torch.tensor([t_step], dtype=torch.float64, device=rdev)
     if world > 1:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     t_step = float(t_max.item())
@@ -522,7 +531,7 @@ def main():
         surv_res = int(D.lengths[surv].sum()) if ns else 0
     else:
         ns, surv_res = (n, res_local) if args.stage == "vit" else (0, 0)
-    tot = torch.tensor([res_local, surv_res, ns, n], dtype=torch.float64, device=dev)
+    tot = torch.tensor([res_local, surv_res, ns, n], dtype=torch.float64, device=rdev)
     if world > 1:
         dist.all_reduce(tot)
     res_all, surv_all, ns_all, n_all = [float(x) for x in tot.tolist()]
@@ -718,8 +727,9 @@ def main():
                        "l2": "flushed (256 MiB write) before every timed step, outside its events",
                        "launch": "CUDA graph of the stage (captured once), replayed per step" if graph is not None
                                  else "eager calls",
-                       "parallelism": "db-shard x%d (snake length-balanced, %s scaling), NCCL all_gather of results"
-                                      % (world, args.scaling),
+                       "parallelism": "db-shard x%d (snake length-balanced, %s scaling), %s all_gather of results"
+                                      % (world, args.scaling, "NCCL" if args.backend == "nccl" else
+                                         "gloo (host-staged, test of the N > 1 path)"),
                        "tuning": args.tune or None},
             "stages": {"msv_kernel_ms": round(msv_ms, 4) if msv_ms > 0 else None,
                        "msv_gcups": round(msv_gcups, 2) if msv_gcups else None,

@@ -61,11 +61,13 @@ class Gatherer:
     exchange   : False builds the static buffers without any collective (one process playing
                  every rank in turn: ``local`` gives the slices all_gather_into_tensor would
                  concatenate in rank order -- the one-GPU proof of the sharded path)
+    stage_host : run the collectives on host copies (gloo tests of the N > 1 path with several
+                 ranks on one GPU; NCCL is the product path)
     """
 
-    def __init__(self, n_global: int, world: int, global_ids, group=None, exchange: bool = True):
+    def __init__(self, n_global: int, world: int, global_ids, group=None, exchange: bool = True,
+                 stage_host: bool = False):
         import torch
-        import torch.distributed as dist
         self.world, self.group = world, group
         self.nmax = max(shard_sizes(n_global, world))
         dev = global_ids.device
@@ -80,10 +82,20 @@ class Gatherer:
         self.gid_pad[:self.n_local] = self.gid_local
         self.gids = torch.empty(world * self.nmax, dtype=torch.int64, device=dev)
         self.exchange = exchange
+        self.stage_host = stage_host
         if world > 1 and exchange:
-            dist.all_gather_into_tensor(self.gids, self.gid_pad, group=group)   # once: the shard map is static
+            self._all_gather(self.gids, self.gid_pad)   # once: the shard map is static
         else:
             self.gids[:self.nmax].copy_(self.gid_pad)
+
+    def _all_gather(self, out, inp):
+        import torch.distributed as dist
+        if self.stage_host:
+            o = out.cpu()
+            dist.all_gather_into_tensor(o, inp.cpu(), group=self.group)
+            out.copy_(o)
+        else:
+            dist.all_gather_into_tensor(out, inp, group=self.group)
 
     def local(self, msv_raw, vit_raw, flags, survivor_ids, n_survivors):
         """This rank's padded slices (device ops only): result words and global survivor ids."""
@@ -97,14 +109,13 @@ class Gatherer:
     def __call__(self, msv_raw, vit_raw, flags, survivor_ids, n_survivors):
         """Gather every rank's results; returns device views words [world, nmax],
         gids [world, nmax], counts [world], surv [world, nmax] (first counts[r] valid)."""
-        import torch.distributed as dist
         if not self.exchange:
             raise RuntimeError("Gatherer(exchange=False) has no collective step")
         pad, sv, ns = self.local(msv_raw, vit_raw, flags, survivor_ids, n_survivors)
         if self.world > 1:
-            dist.all_gather_into_tensor(self.words, pad, group=self.group)
-            dist.all_gather_into_tensor(self.counts, ns, group=self.group)
-            dist.all_gather_into_tensor(self.surv, sv, group=self.group)
+            self._all_gather(self.words, pad)
+            self._all_gather(self.counts, ns)
+            self._all_gather(self.surv, sv)
         else:
             self.words.copy_(pad)
             self.counts.copy_(ns)
