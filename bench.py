@@ -401,7 +401,7 @@ def main():
     ap.add_argument("--no-configs", action="store_true", help="skip the configs 2/4/5 leg (N = 1)")
     ap.add_argument("--no-graph", action="store_true", help="launch the step eagerly in the timed region")
     ap.add_argument("--batch", type=int, default=64, help="profiles of the f4 batch leg (0 = skip)")
-    ap.add_argument("--cpu-sample-every", type=int, default=0, help="default: 2 (pipeline, msv), 23 (vit)")
+    ap.add_argument("--cpu-sample-every", type=int, default=0, help="default: 1 (pipeline, msv), 23 (vit)")
     ap.add_argument("--ref-sample", type=int, default=100000)
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo + --one-device: exercise the N > 1 path with every rank on cuda:0 (tests only)")
@@ -413,7 +413,7 @@ def main():
     args.stage = args.stage or STAGE_OF[args.config]
     args.scaling = args.scaling or SCALING_OF[args.config]
     if not args.cpu_sample_every:
-        args.cpu_sample_every = 23 if args.stage == "vit" else 2   # ~10 s of oracle work on 16 cores
+        args.cpu_sample_every = 23 if args.stage == "vit" else 1   # ~6-10 s of oracle work on 16 cores
 
     rank, world, local = env_rank()
     if args.one_device:
@@ -582,8 +582,10 @@ def main():
         roofline["survey_8d_msv_ratio"] = round(msv_gcups * 1e9 / (p_int * 1e12 / 2), 3) if msv_gcups else None
     roofline["alu"]["peak_source"] = "%s sm_max_mhz x %d SMs x %d lanes/clk (ALU pipe, measured profiles/intpeak_r01.txt)" \
                                      % (src, nsm, ALU_LANES_PER_CLK_SM)
-    ek = evf.get("vit_cpair2_kernel" if args.stage == "vit" and q["vit_pair_lanes"] == 64 else
-                  "msv_fast_kernel" if args.stage != "vit" else "-", {})
+    # DRAM traffic of the captured launch: only for the workloads the ncu captures ran (config 3's
+    # MSV kernel, config 4's Viterbi kernel); other workloads report null
+    ek = evf.get("vit_cpair2_kernel" if args.stage == "vit" and args.config == 4 and q["vit_pair_lanes"] == 64
+                 else "msv_fast_kernel" if args.stage != "vit" and args.config == 3 else "-", {})
     tb, tsrc = ek.get("dram_bytes_per_launch"), ek.get("dram_source")
     roofline["traffic"] = tb
     roofline["traffic_unit"] = "bytes/launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)"
