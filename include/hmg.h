@@ -19,9 +19,12 @@
  *   - Compute calls are asynchronous and stream-ordered on `stream`
  *     (a cudaStream_t passed as void*, NULL = legacy default stream).  They
  *     return after enqueueing; CUDA launch errors map to HMG_ECUDA.
- *   - Handles are immutable after creation (internal per-F threshold caches
- *     are guarded) and may be used from several streams; one handle must not
- *     be destroyed while work using it is in flight.
+ *   - Handles are immutable after creation (the per-F threshold tables a
+ *     profile builds on first use are added under a lock and never freed or
+ *     replaced before hmg_profile_destroy, so calls on other streams and CUDA
+ *     graphs that captured them stay valid) and may be used from several
+ *     streams; one handle must not be destroyed while work using it is in
+ *     flight.
  *   - Sequence indices ("caller order") are positions 0..nseq-1 in the arrays
  *     given to hmg_db_create.  The DB is internally sorted by length
  *     (descending) for scheduling; all outputs are in caller order.

@@ -195,3 +195,17 @@ def test_tuning_api():
     hmg.clear_tuning()
     src = open(os.path.join(os.path.dirname(__file__), "..", "paper_conf_ipps_jiangg15_b200", "csrc", "host.cu")).read()
     assert "getenv" not in src
+
+
+def test_tuning_knobs_documented():
+    """Every knob the library accepts is listed in include/hmg.h (hmg_set_tuning's contract)."""
+    here = os.path.dirname(__file__)
+    src = open(os.path.join(here, "..", "paper_conf_ipps_jiangg15_b200", "csrc", "host.cu")).read()
+    names = re.findall(r'"([A-Z0-9_]+)"', src[src.index("kTuneNames[]"):src.index("};", src.index("kTuneNames[]"))])
+    hdr = open(os.path.join(here, "..", "include", "hmg.h")).read()
+    doc = hdr[hdr.index("hmg_set_tuning") - 2000:hdr.index("hmg_set_tuning")]
+    assert len(names) > 20
+    for n in names:
+        assert n in doc, n
+        hmg.set_tuning(n, 0)
+    hmg.clear_tuning()
