@@ -147,6 +147,8 @@ struct hmg_profile {
   int pair_G = 0, pair_Q = 0;       // >0: s16x2 pair kernel vit_pair_kernel<G, Q> first, the above re-scores
   bool pair_scan = false;           // pair kernel: max-plus scan Lazy-F (G = 32 only; HMG_VIT_SCAN)
   int pair_SG2 = 0;                 // >0: W = 2 without the per-row barrier, vit_cpair2_kernel<pair_Q, pair_SG2>
+  int pair_wide = 0;                // one warp per sequence, Q <= 32: vit_wide_kernel<pair_Q, tm> (pair_G = 32);
+                                    // 1: transitions in shared memory, 2: in tensor memory
   int pair_W = 0, pair_SG = 1;      // >0: block pair kernel vit_cpair_kernel<pair_W, pair_Q, pair_SG>
                                     //     (pair_G = 32 W; pair_SG sequences per block share its table)
   int tbm_min = 0, rmax = 0;        // pair kernel window: min_k tBM_k, max(0, max_{x,k} rsc)
@@ -229,6 +231,9 @@ cudaError_t launch_vit_cpair(int W, int SG, int Q, const VitArgs& a, cudaStream_
 size_t vit_cpair_smem(int W, int SG, int Q);
 bool vit_cpair_available(int W, int SG, int Q);
 cudaError_t launch_vit_cpair2(int SG, int Q, const VitArgs& a, cudaStream_t st, int* ok);
+cudaError_t launch_vit_wide(int Q, bool tm, const VitArgs& a, cudaStream_t st, int* ok);
+bool vit_wide_available(int Q);
+size_t vit_wide_smem(int Q, bool tm);
 size_t vit_cpair2_smem(int SG, int Q);
 bool vit_cpair2_available(int SG, int Q);
 int vit_pair_q_max();

@@ -179,7 +179,7 @@ const char* const kTuneNames[] = {
     "MSV_G", "VIT_G", "MSV_LLONG", "NO_LONG_LANE", "FWD_QMAX", "FWD_W", "FWD_S", "VIT_CTA", "VIT_CTA_W",
     "VIT_GENERIC", "NO_VIT_PAIR", "VIT_PAIR_G", "VIT_PAIR_CTA", "VIT_SCAN", "VIT_PAIR_W", "VIT_PAIR_SG",
     "VIT_CPAIR2", "LONG_S32", "PIPE_LLONG", "PIPE_CHUNK", "UPLOAD_PARTS", "UPLOAD_FIRST_PERMILLE",
-    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS"};
+    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS", "VIT_WIDE"};
 std::mutex g_tune_mu;
 std::map<std::string, int> g_tune;
 
@@ -656,7 +656,9 @@ hmg_status run_vit(const hmg_profile* p, const hmg_db* db, const int32_t* list, 
     b.redo_list = redo;
     b.redo_count = ctr + 1;
     int ok = 0;
-    if (p->pair_SG2 > 0) {
+    if (p->pair_wide) {
+      if ((e = launch_vit_wide(p->pair_Q, p->pair_wide == 2, b, st, &ok))) return cuda_status(e);
+    } else if (p->pair_SG2 > 0) {
       if ((e = launch_vit_cpair2(p->pair_SG2, p->pair_Q, b, st, &ok))) return cuda_status(e);
     } else if (p->pair_W > 0) {
       if ((e = launch_vit_cpair(p->pair_W, p->pair_SG, p->pair_Q, b, st, &ok))) return cuda_status(e);
@@ -960,6 +962,17 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
         const int sg2 = tune_int("VIT_CPAIR2", 2);
         if (p->pair_W == 2 && sg2 > 0 && vit_cpair2_available(sg2, qq) && vit_cpair2_smem(sg2, qq) <= (size_t)smax)
           p->pair_SG2 = sg2;
+        // one warp per sequence, transitions in shared (VIT_WIDE = 1) or tensor memory (2)
+        // (vit_wide.cuh): 64 Q4 >= M
+        const int q4 = ((M + 63) / 64 + 3) / 4 * 4;
+        const int wide = tune_int("VIT_WIDE", 0);
+        if ((wide == 1 || wide == 2) && vit_wide_available(q4) && vit_wide_smem(q4, wide == 2) <= (size_t)smax) {
+          p->pair_wide = wide;
+          p->pair_W = 0;
+          p->pair_SG2 = 0;
+          p->pair_G = 32;
+          p->pair_Q = q4;
+        }
       }
     }
   }
@@ -1017,7 +1030,7 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   }
   // pipeline long lane: whole-warp Viterbi with the pair lane (the pair tables when G = 32, models
   // up to 1024 nodes) or the s32 latency lane (models up to 512 nodes)
-  const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !tune_int("LONG_S32", 0);
+  const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !p->pair_wide && !tune_int("LONG_S32", 0);
   if (st == HMG_OK && tsc && (lpair || M <= 512) && !tune_int("NO_LONG_LANE", 0)) {
     const int QL = long_msv_q(M);
     auto tm = msv_table(*p, 32, QL);

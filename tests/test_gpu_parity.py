@@ -606,7 +606,7 @@ def test_pipeline_many_survivors(M):
 
 
 @pytest.mark.parametrize("M", [2, 3, 64, 300, 513, 1024, 1025, 1500, 2048, 2600, 4000])
-@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t"])
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t", "wide", "wide_tm"])
 def test_vit_block_pair_kernel(M, W, tune):
     """Block-per-sequence pair kernel (W warps per row, 2 cells per register, closed-form carries
     across virtual warps); forced for small M with tuning VIT_PAIR_CTA, used by default above 1024.
@@ -616,6 +616,9 @@ def test_vit_block_pair_kernel(M, W, tune):
     if W in ("2b", "2t"):
         tune("VIT_CPAIR2", "0" if W == "2b" else "23")
         W = 2
+    if W in ("wide", "wide_tm"):                     # one warp, transitions in shared / tensor memory (vit_wide.cuh)
+        tune("VIT_WIDE", 1 if W == "wide" else 2)
+        W = 1
     tune("VIT_PAIR_W", str(W))
     rng = np.random.default_rng(M * 7 + W)
     for dd in [(7.0, 3.0), (1.0, 9.0)]:
@@ -628,7 +631,7 @@ def test_vit_block_pair_kernel(M, W, tune):
         assert np.array_equal(got, oracle.vit_db(oracle.VitProfile(prof.msc, prof.tsc), dsq, off)), dd
 
 
-@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t"])
+@pytest.mark.parametrize("W", [2, 4, 8, 16, "2b", "2t", "wide", "wide_tm"])
 def test_vit_block_pair_delete_chains_and_exits(W, tune):
     """D->D chains across every virtual-warp boundary (low halves -> high halves), strong hits that
     re-base the window or overflow, and gap-only sequences handed to the s32 kernel."""
@@ -636,6 +639,9 @@ def test_vit_block_pair_delete_chains_and_exits(W, tune):
     if W in ("2b", "2t"):
         tune("VIT_CPAIR2", "0" if W == "2b" else "23")
         W = 2
+    if W in ("wide", "wide_tm"):                     # one warp, transitions in shared / tensor memory (vit_wide.cuh)
+        tune("VIT_WIDE", 1 if W == "wide" else 2)
+        W = 1
     tune("VIT_PAIR_W", str(W))
     for M in (40, 700, 2000):
         rng = np.random.default_rng(M + W)

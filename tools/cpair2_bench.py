@@ -14,8 +14,12 @@ D = hmg.Database(dsq, off)
 prof = synth.make_profile(M, 1000 + M)
 hmg.hmg_set_stage_timing(True)
 ref = None
-for sg in ("0", "2", "12", "22", "23"):
-    hmg.set_tuning("VIT_CPAIR2", int(sg))
+for sg in ("0", "2", "wide", "wide_tm"):
+    hmg.clear_tuning()
+    if sg in ("wide", "wide_tm"):
+        hmg.set_tuning("VIT_WIDE", 1 if sg == "wide" else 2)
+    else:
+        hmg.set_tuning("VIT_CPAIR2", int(sg))
     P = hmg.Profile(prof.msc, prof.tsc)
     raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
     ts = []
@@ -24,6 +28,6 @@ for sg in ("0", "2", "12", "22", "23"):
         ts.append(hmg.hmg_stage_times()["vit_kernel"])
     best = min(ts[1:])
     ref = raw.clone() if ref is None else ref
-    print(json.dumps({"M": M, "N": N, "kernel": "cpair (barrier)" if sg == "0" else "cpair2 var=%s (10 TSM + SG)" % sg,
+    print(json.dumps({"M": M, "N": N, "kernel": "cpair (barrier)" if sg == "0" else "wide (one warp, smem)" if sg == "wide" else "wide (one warp, TMEM)" if sg == "wide_tm" else "cpair2 var=%s (10 TSM + SG)" % sg,
                       "ms": round(best, 3), "gcups": round(M * D.residues / best / 1e6, 1),
                       "redo": hmg.hmg_stage_counts()["vit_pair_redo"], "same": bool(torch.equal(ref, raw))}), flush=True)

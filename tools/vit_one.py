@@ -1,5 +1,5 @@
 """One Viterbi-filter call over a config-2-shaped DB for a given M (for ncu captures):
-python tools/vit_one.py M [nseq]"""
+python tools/vit_one.py M [nseq] [KNOB=VALUE ...]  (tuning knobs, include/hmg.h)"""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -7,6 +7,9 @@ from paper_conf_ipps_jiangg15_b200 import build, hmg, synth
 build.build()
 M = int(sys.argv[1])
 N = int(sys.argv[2]) if len(sys.argv) > 2 else 100000
+for kv in sys.argv[3:]:
+    k, v = kv.split("=")
+    hmg.set_tuning(k, int(v))
 prof = synth.make_profile(M, 1000 + M)
 db = synth.make_db(N, 5.60, 0.75, 12)
 dsq, off = db.materialize()
