@@ -75,6 +75,15 @@ def load_evidence():
 
 
 STAGE_OF = {1: "pipeline", 2: "msv", 3: "pipeline", 4: "vit", 5: "pipeline"}
+# hmg_quant.vit_pair_kernel -> (evidence key in profiles/kernel_evidence_r02.json, kernel name)
+VIT_KERNELS = {1: ("vit_pair_kernel", "vit_pair_kernel"), 2: ("vit_cpair_kernel", "vit_cpair_kernel"),
+               3: ("vit_cpair2_kernel", "vit_cpair2_kernel"), 4: ("vit_wide_kernel_smem", "vit_wide_kernel<Q,0>"),
+               5: ("vit_wide_kernel", "vit_wide_kernel<Q,1> (TMEM transitions)")}
+
+
+def vit_kernel(q):
+    key, name = VIT_KERNELS.get(q["vit_pair_kernel"], ("-", "s32 Viterbi kernel"))
+    return key, "%s, %d lanes x %d registers" % (name, q["vit_pair_lanes"], q["vit_pair_regs"])
 SCALING_OF = {1: "weak", 2: "weak", 3: "weak", 4: "strong", 5: "strong"}
 
 
@@ -336,18 +345,19 @@ def configs_leg(args, dev, stream, flush, p_int, ev_file):
                 raw = torch.empty(n, dtype=torch.int16, device=dev)
                 pas = torch.empty(n, dtype=torch.uint8, device=dev)
                 fn = lambda: hmg.hmg_viterbi(P, D2, raw, pass_=pas, F2=args.F2, stream=stream)
-                key, ops, stage = "vit_cpair2_kernel", VIT_ALU_OPS_PER_CELL, "vit_kernel"
+                key, ops, stage = None, VIT_ALU_OPS_PER_CELL, "vit_kernel"
             ms = timed_ms(fn, stream, flush, 3 if cfg == 2 else 2)
             kms = hmg.hmg_stage_times()[stage]
             cells = c["M"] * D2.residues
             q = P.quant()
+            if key is None:
+                key, vlabel = vit_kernel(q)
             out.append({"config": cfg, "stage": "msv" if cfg == 2 else "vit", "M": c["M"], "nseq": n,
                         "residues": D2.residues, "ms": round(ms, 3), "gcups": round(cells / ms / 1e6, 1),
                         "kernel_ms": round(kms, 3), "kernel_gcups": round(cells / kms / 1e6, 1),
                         "roofline": kernel_roofline(ev_file, key, cells, kms, p_int, ops,
                                                     ("msv_fast_kernel G=%d Q=%d" % (q["msv_lanes"], q["msv_regs"]))
-                                                    if cfg == 2 else
-                                                    ("vit_cpair2_kernel Q=%d" % q["vit_pair_regs"]))})
+                                                    if cfg == 2 else vlabel)})
             print("configs leg: config %d %.3f ms" % (cfg, ms), file=sys.stderr, flush=True)
         del D2
         c5 = synth.CONFIGS[5]
@@ -567,9 +577,8 @@ def main():
     evf = load_evidence()
     q = P.quant()
     if args.stage == "vit":
-        vkey = "vit_cpair2_kernel" if q["vit_pair_lanes"] == 64 else "vit_pair_kernel"
-        roofline = kernel_roofline(evf, vkey, M * surv_res, vit_ms, p_int, VIT_ALU_OPS_PER_CELL,
-                                   "Viterbi kernel (pair lanes %d x %d registers)" % (q["vit_pair_lanes"], q["vit_pair_regs"]))
+        vkey, vlabel = vit_kernel(q)
+        roofline = kernel_roofline(evf, vkey, M * surv_res, vit_ms, p_int, VIT_ALU_OPS_PER_CELL, vlabel)
         roofline["kernel_share_of_step"] = round(vit_ms / t_step, 4)
     else:
         roofline = kernel_roofline(evf, "msv_fast_kernel", M * res_local, msv_ms, p_int, MSV_ALU_OPS_PER_CELL,
@@ -584,7 +593,7 @@ def main():
                                      % (src, nsm, ALU_LANES_PER_CLK_SM)
     # DRAM traffic of the captured launch: only for the workloads the ncu captures ran (config 3's
     # MSV kernel, config 4's Viterbi kernel); other workloads report null
-    ek = evf.get("vit_cpair2_kernel" if args.stage == "vit" and args.config == 4 and q["vit_pair_lanes"] == 64
+    ek = evf.get(vit_kernel(q)[0] if args.stage == "vit" and args.config == 4
                  else "msv_fast_kernel" if args.stage != "vit" and args.config == 3 else "-", {})
     tb, tsrc = ek.get("dram_bytes_per_launch"), ek.get("dram_source")
     roofline["traffic"] = tb

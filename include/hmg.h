@@ -85,6 +85,11 @@ typedef struct {
   int fwd_seqs_per_block;           /* Forward kernel: sequences per block sharing the staged table */
   int fwd_lanes;                    /* Forward kernel: threads per sequence (8 = sub-warp lane groups
                                        for M <= 32; else 32 x fwd_warps) */
+  int vit_pair_kernel;              /* which s16x2 Viterbi kernel (DESIGN.md 4.3b-d): 0 none, 1 lane groups
+                                       (vit_pair), 2 warps joined per row (vit_cpair), 3 two warps
+                                       without a row barrier (vit_cpair2), 4 one warp with the
+                                       transitions in shared memory (vit_wide), 5 one warp with the
+                                       transitions in tensor memory (vit_wide, tcgen05.ld) */
 } hmg_quant;
 
 /* ---------------------------------------------------------------- profile */
@@ -266,7 +271,8 @@ hmg_status hmg_prepare_thresholds(const hmg_profile* p, double F1, double F2, in
  * Knobs (int): MSV_G, VIT_G, MSV_LLONG, NO_LONG_LANE, FWD_QMAX, FWD_W, FWD_S, VIT_CTA, VIT_CTA_W,
  * VIT_GENERIC, NO_VIT_PAIR, VIT_PAIR_G, VIT_PAIR_CTA, VIT_SCAN, VIT_PAIR_W, VIT_PAIR_SG,
  * VIT_CPAIR2, LONG_S32, PIPE_LLONG, PIPE_CHUNK, UPLOAD_PARTS, UPLOAD_FIRST_PERMILLE, UPLOAD_GROW,
- * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS, VIT_WIDE.  Geometry knobs take effect at profile / DB
+ * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS, VIT_WIDE (0 off, 1 shared, 2 tensor memory).
+ * Geometry knobs take effect at profile / DB
  * creation, schedule knobs at the next call.  HMG_EINVAL for an unknown name. */
 hmg_status hmg_set_tuning(const char* name, int value);
 /* Remove one override (name) or all of them (name == NULL). */

@@ -962,10 +962,12 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
         const int sg2 = tune_int("VIT_CPAIR2", 2);
         if (p->pair_W == 2 && sg2 > 0 && vit_cpair2_available(sg2, qq) && vit_cpair2_smem(sg2, qq) <= (size_t)smax)
           p->pair_SG2 = sg2;
-        // one warp per sequence, transitions in shared (VIT_WIDE = 1) or tensor memory (2)
-        // (vit_wide.cuh): 64 Q4 >= M
+        // one warp per sequence, transitions in tensor (VIT_WIDE = 2) or shared memory (1)
+        // (vit_wide.cuh): 64 Q4 >= M.  Default from profiles/wide_r02zc.jsonl (100k sequences):
+        // M = 2048 TMEM 2 775 GCUPS vs shared 2 233 vs two warps 2 204; M = 1500 2 622 / 2 268 /
+        // 1 847; M = 1100 (Q4 = 20) 2 227 / 2 318 / 1 839
         const int q4 = ((M + 63) / 64 + 3) / 4 * 4;
-        const int wide = tune_int("VIT_WIDE", 0);
+        const int wide = tune_int("VIT_WIDE", q4 >= 24 ? 2 : 1);
         if ((wide == 1 || wide == 2) && vit_wide_available(q4) && vit_wide_smem(q4, wide == 2) <= (size_t)smax) {
           p->pair_wide = wide;
           p->pair_W = 0;
@@ -1167,6 +1169,10 @@ hmg_status hmg_profile_quant(const hmg_profile* p, hmg_quant* q) {
   q->vit_nodes = p->vit_generic ? 0 : p->vit_Q;
   q->vit_pair_lanes = p->pair_G;
   q->vit_pair_regs = p->pair_Q;
+  q->vit_pair_kernel = p->pair_G == 0 ? 0
+                       : p->pair_wide ? 3 + p->pair_wide
+                       : p->pair_SG2 > 0 ? 3
+                       : p->pair_W > 0 ? 2 : 1;
   q->fwd_warps = p->fwd_W;
   q->fwd_lanes = p->fwd_T;
   q->fwd_nodes = p->fwd_Q;

@@ -33,7 +33,7 @@ class hmg_quant(ctypes.Structure):
                 ("msv_regs", c_int), ("vit_lanes", c_int), ("vit_nodes", c_int),
                 ("vit_pair_lanes", c_int), ("vit_pair_regs", c_int),
                 ("fwd_warps", c_int), ("fwd_nodes", c_int), ("fwd_rows_smem", c_int),
-                ("fwd_seqs_per_block", c_int), ("fwd_lanes", c_int)]
+                ("fwd_seqs_per_block", c_int), ("fwd_lanes", c_int), ("vit_pair_kernel", c_int)]
 
 
 # name -> (restype, argtypes), exactly the declarations of include/hmg.h

@@ -46,3 +46,11 @@ def test_workload_sharding(scaling, world, n):
     c, prof, db = bench.workload(A, world)
     assert prof.M == 400
     assert db.N == (n * world if scaling == "weak" else n)
+
+
+def test_bench_names_the_viterbi_kernel():
+    """hmg_quant.vit_pair_kernel picks the evidence entry and the label of the Viterbi roofline."""
+    for kind in range(1, 6):
+        key, label = bench.vit_kernel({"vit_pair_kernel": kind, "vit_pair_lanes": 32, "vit_pair_regs": 32})
+        assert key == bench.VIT_KERNELS[kind][0] and "32 lanes" in label
+    assert bench.vit_kernel({"vit_pair_kernel": 0, "vit_pair_lanes": 0, "vit_pair_regs": 0})[0] == "-"

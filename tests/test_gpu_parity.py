@@ -441,19 +441,23 @@ def _stratified(lengths, n, rng):
     return np.unique(np.concatenate([rng.choice(pp, n // 10, replace=False) for pp in parts]))
 
 
-def test_viterbi_config4_full_size_sampled():
+@pytest.mark.parametrize("kernel", ["wide_tm", "cpair2"])
+def test_viterbi_config4_full_size_sampled(kernel, tune):
     """BASELINE config 4 at full size in the bench launch configuration: the Viterbi filter
-    (Lazy-F) over every one of the 550k Swiss-Prot-shaped sequences at M = 2048 (the two-warp
-    kernel, M up to 2405 P:816-818).  The oracle checks a 2k length-stratified sample,
-    the 50 longest sequences (L up to 35,213) and the pass flags there; planted homologs (strong
-    hits that re-base the 16-bit window) are checked on a second 20k-sequence DB."""
+    (Lazy-F) over every one of the 550k Swiss-Prot-shaped sequences at M = 2048 (M up
+    to 2405 P:816-818), with the bench's kernel (one warp per sequence, transitions in tensor
+    memory) and the two-warp one.  The oracle checks a 2k length-stratified sample, the 50 longest
+    sequences (L up to 35,213) and the pass flags there; planted homologs (strong hits that re-base
+    the 16-bit window) are checked on a second 20k-sequence DB."""
+    if kernel == "cpair2":
+        tune("VIT_WIDE", 0)
     c = synth.CONFIGS[4]
     prof = synth.make_profile(c["M"], c["pseed"])
     db = synth.make_db(c["N"], c["mu_ln"], c["sigma"], c["dseed"])
     dsq, off = db.materialize()
     ev = _calibrate(prof)
     p = hmg.Profile(prof.msc, prof.tsc, ev=ev)
-    assert p.quant()["vit_pair_lanes"] == 64                       # the two-warp pair kernel
+    assert p.quant()["vit_pair_kernel"] == (5 if kernel == "wide_tm" else 3)
     D = hmg.Database(dsq, off)
     raw = torch.full((D.nseq,), -12345, dtype=torch.int16, device="cuda")
     pas = torch.zeros(D.nseq, dtype=torch.uint8, device="cuda")
@@ -611,7 +615,9 @@ def test_vit_block_pair_kernel(M, W, tune):
     """Block-per-sequence pair kernel (W warps per row, 2 cells per register, closed-form carries
     across virtual warps); forced for small M with tuning VIT_PAIR_CTA, used by default above 1024.
     W = 2 runs the kernel without a per-row barrier (vit_cpair2.cuh); "2b" the barrier kernel;
-    "2t" the barrier-free kernel with four transition vectors in shared memory (3 sequences/block)."""
+    "2t" the barrier-free kernel with four transition vectors in shared memory (3 sequences/block);
+    "wide" / "wide_tm" one warp per sequence with the transitions in shared / tensor memory
+    (vit_wide.cuh, the default above 1024 nodes)."""
     tune("VIT_PAIR_CTA", "1")
     if W in ("2b", "2t"):
         tune("VIT_CPAIR2", "0" if W == "2b" else "23")
@@ -619,6 +625,8 @@ def test_vit_block_pair_kernel(M, W, tune):
     if W in ("wide", "wide_tm"):                     # one warp, transitions in shared / tensor memory (vit_wide.cuh)
         tune("VIT_WIDE", 1 if W == "wide" else 2)
         W = 1
+    else:
+        tune("VIT_WIDE", 0)
     tune("VIT_PAIR_W", str(W))
     rng = np.random.default_rng(M * 7 + W)
     for dd in [(7.0, 3.0), (1.0, 9.0)]:
@@ -642,6 +650,8 @@ def test_vit_block_pair_delete_chains_and_exits(W, tune):
     if W in ("wide", "wide_tm"):                     # one warp, transitions in shared / tensor memory (vit_wide.cuh)
         tune("VIT_WIDE", 1 if W == "wide" else 2)
         W = 1
+    else:
+        tune("VIT_WIDE", 0)
     tune("VIT_PAIR_W", str(W))
     for M in (40, 700, 2000):
         rng = np.random.default_rng(M + W)

@@ -209,3 +209,23 @@ def test_tuning_knobs_documented():
         assert n in doc, n
         hmg.set_tuning(n, 0)
     hmg.clear_tuning()
+
+
+@pytest.mark.parametrize("M,kind", [(40, 1), (400, 1), (1024, 1), (1100, 4), (1500, 5), (2048, 5), (3000, 2)])
+def test_viterbi_kernel_choice(M, kind):
+    """Which s16x2 Viterbi kernel a profile gets (hmg_quant.vit_pair_kernel, DESIGN.md 4.3b-d):
+    lane groups up to 1024 nodes, one warp per sequence above (transitions in shared memory up to
+    1280 nodes, in tensor memory to 2048), warps joined per row beyond; VIT_WIDE = 0 restores the
+    two-warp kernel."""
+    prof = synth.make_profile(M, 77 + M)
+    q = hmg.Profile(prof.msc, prof.tsc, device=-1).quant()
+    assert q["vit_pair_kernel"] == kind
+    assert 2 * q["vit_pair_lanes"] * q["vit_pair_regs"] >= M
+    if kind in (4, 5):
+        assert q["vit_pair_lanes"] == 32
+        hmg.set_tuning("VIT_WIDE", 0)
+        try:
+            assert hmg.Profile(prof.msc, prof.tsc, device=-1).quant()["vit_pair_kernel"] in (2, 3)
+        finally:
+            hmg.clear_tuning()
+

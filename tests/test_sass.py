@@ -24,7 +24,9 @@ KERNELS = {
     "_ZN3hmg18msv_fast_kernel_mbILi8ELi26ELi3EEEvNS_7MsvArgsE": (150, 60),      # config 3 MSV (M = 400)
     "_ZN3hmg15msv_fast_kernelILi8ELi13EEEvNS_7MsvArgsE": (60, 30),             # config 2 MSV (M = 200)
     "_ZN3hmg15vit_pair_kernelILi32ELi7ELb0EEEvNS_7VitArgsE": (40, 3),           # config 3 Viterbi stage
-    "_ZN3hmg17vit_cpair2_kernelILi16ELi2ELi0EEEvNS_7VitArgsE": (120, 5),        # config 4 Viterbi (M = 2048)
+    "_ZN3hmg17vit_cpair2_kernelILi16ELi2ELi0EEEvNS_7VitArgsE": (120, 5),        # two-warp Viterbi (M <= 2048)
+    "_ZN3hmg15vit_wide_kernelILi32ELb1EEEvNS_7VitArgsE": (300, 10),            # config 4 Viterbi (M = 2048, TMEM)
+    "_ZN3hmg15vit_wide_kernelILi20ELb0EEEvNS_7VitArgsE": (300, 10),            # 1024 < M <= 1280 (shared memory)
     "_ZN3hmg19msv_multi_kernel_mbILi8ELi26ELi3EEEvNS_12MsvMultiArgsE": (100, 50),  # f4 batch MSV
     "_ZN3hmg22pipe_long_vpair_kernelILi7EEEvNS_8LongArgsE": (40, 3),           # config 3 long lane
 }
@@ -55,3 +57,15 @@ def test_hot_kernel_is_native_dpx(lib_path, fn):
     assert max3 >= lo3, (fn, max3)
     bad = [l.strip() for l in lines if any(p.search(l) for p in EMULATION)]
     assert not bad, bad[:5]
+
+
+def test_wide_kernel_reads_transitions_from_tensor_memory(lib_path):
+    """vit_wide_kernel<Q, true> streams the transition vectors with tcgen05.ld
+    (SASS LDTM), two loads per chunk of four registers in the M / I sweep and one in the D chain,
+    and allocates / frees its TMEM columns (UTCATOMSWS)."""
+    lines = _sass(lib_path, "_ZN3hmg15vit_wide_kernelILi32ELb1EEEvNS_7VitArgsE")
+    ldtm = sum("LDTM" in l for l in lines)
+    assert ldtm >= 3 * 8, ldtm
+    assert any("UTCATOMSWS" in l for l in lines)
+    smem = _sass(lib_path, "_ZN3hmg15vit_wide_kernelILi32ELb0EEEvNS_7VitArgsE")
+    assert not any("LDTM" in l for l in smem)

@@ -19,6 +19,7 @@ for sg in ("0", "2", "wide", "wide_tm"):
     if sg in ("wide", "wide_tm"):
         hmg.set_tuning("VIT_WIDE", 1 if sg == "wide" else 2)
     else:
+        hmg.set_tuning("VIT_WIDE", 0)
         hmg.set_tuning("VIT_CPAIR2", int(sg))
     P = hmg.Profile(prof.msc, prof.tsc)
     raw = torch.zeros(D.nseq, dtype=torch.int16, device="cuda")
