@@ -22,6 +22,7 @@
 // where the vote fires.  Valid iff bias < 66 + tbm (host check); otherwise the
 // exact kernel runs.
 #pragma once
+#include <type_traits>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -129,21 +130,30 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
   const int nw = (L + 5) / 6;
   const int tjb = valid ? a.tjb[L] : 0;
 
-  int xJ = 0;
-  bool ovf = false;
-  int Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
-  uint32_t B2 = (uint32_t)Bp * 0x10001u;
-  uint32_t thrv = valid ? (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u : 0u;   // 0: never fires
-
+  int xJ;
+  bool ovf;
+  int Bp;
+  uint32_t B2, thrv, R;
   uint32_t t[Q];
+  auto reset = [&]() {
+    xJ = 0;
+    ovf = false;
+    Bp = min(max(kBaseB - tjb - tbm, 0) + bias, 255);
+    B2 = (uint32_t)Bp * 0x10001u;
+    thrv = valid ? (uint32_t)(0x8000 - msv_thr(xJ, bias)) * 0x10001u : 0u;   // 0: never fires
 #pragma unroll
-  for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
-  uint32_t R = B2;
+    for (int q = 0; q < Q; ++q) t[q] = B2;   // row 1: max(0 + bias, B') = B'
+    R = B2;
+  };
 
   const int nqmax = (Lmax + 23) / 24;
-  ResStream rs;
-  rs.init(wp, nw);
-  for (int iq = 0; iq < nqmax; ++iq) {
+  // All rows of the batch.  CHECK: the per-row J->B / overflow vote and update (Alg 1 l.16-20)
+  // after every row; without it (Q > 8, first pass) the rows run branch-free.
+  auto run = [&](auto check_tag) {
+   constexpr bool CHECK = decltype(check_tag)::value;
+   ResStream rs;
+   rs.init(wp, nw);
+   for (int iq = 0; iq < nqmax; ++iq) {
    uint4 w4 = rs.next(iq);
 #pragma unroll 1
    for (int k = 0; k < 4; ++k) {
@@ -209,9 +219,26 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
       }
     } else {
 #pragma unroll
-      for (int j = 0; j < 6; ++j) row((w >> (5 * j)) & 31, true);
+      for (int j = 0; j < 6; ++j) row((w >> (5 * j)) & 31, CHECK);
     }
    }
+   }
+  };
+  reset();
+  if constexpr (Q <= 8) {
+    run(std::true_type{});
+  } else {
+    // Long rows: first the whole batch without the per-row update -- a branch per row pins t[]
+    // to fixed registers, and ptxas then copies all Q of them back after every row (26
+    // IMAD.MOV per row at Q = 26, a third of the kernel's instructions; 9.6% of the kernel's
+    // time, profiles/stage_nocheck_r02zh.jsonl).  With the threshold fixed and R a running max,
+    // that pass is exact unless some cell reached the J->B / overflow threshold; then (rare:
+    // about 0.2% of config-3 sequences) the batch is scored again with the per-row update.
+    run(std::false_type{});
+    if (__any_sync(0xffffffffu, (__vadd2(R, thrv) & 0x80008000u) != 0u)) {
+      reset();
+      run(std::true_type{});
+    }
   }
   // final xJ = max over all cells of (s - 3); R holds max over t = max(s + bias, B')
   uint32_t m = R;
