@@ -300,11 +300,11 @@ hmg_status hmg_stage_counts(int64_t* counts);
 
 /* hmg_db_upload + hmg_pipeline with the upload overlapped: the packed image (host, pinned; from
  * hmg_db_image of this DB) is copied in length-ordered parts on a side stream (a first part of
- * 5% of the residues, then 5 parts of about equal residues; env HMG_UPLOAD_PARTS / _FIRST_PERMILLE
- * / _GROW), each followed by a 4-byte copy that sets its landing flag; ONE MSV launch scores every
- * part, each batch of sequences waiting on its part's flag (the long lane starts with the first
- * part), so the H2D of the later parts hides behind the filter with no kernel boundary per part
- * (HMG_UPLOAD_GATED=0: one MSV launch per part).
+ * 5% of the residues, then 5 parts of about equal residues; tuning knobs UPLOAD_PARTS /
+ * UPLOAD_FIRST_PERMILLE / UPLOAD_GROW, hmg_set_tuning), each part's landing recorded as an event;
+ * one MSV launch per part on a second side stream waits for its part's event only (the long lane
+ * starts after the first part), so the H2D of the later parts hides behind the filter of the
+ * earlier ones.
  * Outputs and results are hmg_pipeline's.  The image must stay valid until the call's work on
  * `stream` has completed. */
 hmg_status hmg_pipeline_upload(const hmg_profile* p, hmg_db* db, const uint32_t* image, double F1, double F2,

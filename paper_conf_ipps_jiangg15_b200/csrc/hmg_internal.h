@@ -20,6 +20,25 @@ constexpr int kBaseW = 12000;   // Viterbi word base (reading R2)
 constexpr int16_t kNegE = -16384;   // "minus infinity" emission / carry of the s16x2 MSV lanes
 constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
 
+// MsvLayout<G, Q> (msv.cuh) for run-time (G, Q): words per residue row (STRIDE), the offsets of the
+// remainder chunks' copy 0 (b2, b1), their copy counts, and the table size in words (WORDS).
+// The host table builder (host.cu msv_table) and the launchers use this; msv.cu checks it
+// against the template for every instantiated geometry.
+struct MsvLayoutRT {
+  int n4, has2, has1, nc2, nc1, b2, b1, roww, ncopy, stride, copy, words;
+  __host__ __device__ constexpr MsvLayoutRT(int G, int Q)
+      : n4(Q / 4), has2(Q % 4 >= 2), has1(Q % 2), nc2(G == 8 ? 2 : 1), nc1(G == 8 ? 4 : (G == 16 ? 2 : 1)),
+        b2(Q / 4 * 4 * G), b1(Q / 4 * 4 * G + (Q % 4 >= 2 ? 2 * G * (G == 8 ? 2 : 1) : 0)),
+        roww(Q / 4 * 4 * G + (Q % 4 >= 2 ? 2 * G * (G == 8 ? 2 : 1) : 0) +
+             (Q % 2 ? G * (G == 8 ? 4 : (G == 16 ? 2 : 1)) : 0)),
+        ncopy(G < 8 ? 8 / G : 1),
+        stride(0), copy(0), words(0) {
+    stride = ncopy > 1 ? (roww + 31) / 32 * 32 : roww;
+    copy = kRows * stride;
+    words = ((ncopy * copy + (ncopy - 1) * 4 * G) + 3) / 4 * 4;
+  }
+};
+
 // ---------------------------------------------------------------- MSV kernel arguments
 
 struct MsvArgs {

@@ -243,40 +243,35 @@ void vit_geometry(int M, int* G, int* Q) {
   *Q = q <= vit_q_max(g) ? q : 0;
 }
 
-// striped MSV table: row x, register q of lane z holds e for nodes z*Q+q+1 (lo), (z+G)*Q+q+1 (hi)
+// striped MSV table: row x, register q of lane z holds e for nodes z*Q+q+1 (lo), (z+G)*Q+q+1 (hi),
+// in the layout of MsvLayout<G, Q> (msv.cuh): 4-word chunks, then the 2-word and 1-word remainder
+// chunks in L.nc2 / L.nc1 per-group copies; G < 8: L.ncopy whole-table copies, rows padded to
+// 128 B, copy k shifted 16*G*k B
 std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
   const int M = p.M;
-  const int ROWW = Q * G;
-  const int n4 = Q / 4, r = Q % 4;
-  auto word_index = [&](int z, int q) {
-    if (q < n4 * 4) return (q / 4) * 4 * G + z * 4 + (q % 4);
-    int b = n4 * 4 * G;
-    int qq = q - n4 * 4;
-    if (r >= 2) {
-      if (qq < 2) return b + z * 2 + qq;
-      b += 2 * G;
-      qq -= 2;
-    }
-    return b + z;
-  };
+  const MsvLayoutRT L(G, Q);
   auto e_of = [&](int x, int node) -> int16_t {   // node 1-based
     if (x >= kAlpha || node > M) return kNegE;
     return (int16_t)(p.bias - (int)p.cost[(size_t)x * M + (node - 1)]);
   };
-  // MsvLayout<G, Q> (msv.cuh): G < 8 -> 8/G copies, rows padded to 128 B, copy k shifted 16*G*k B
-  const int ncopy = G < 8 ? 8 / G : 1;
-  const int stride = ncopy > 1 ? (ROWW + 31) / 32 * 32 : ROWW;
-  const int copy = kRows * stride;
-  std::vector<uint32_t> out((size_t)msv_table_words(G, Q), 0u);
-  for (int k = 0; k < ncopy; ++k)
-    for (int x = 0; x < kRows; ++x)
+  std::vector<uint32_t> out((size_t)L.words, 0u);
+  for (int k = 0; k < L.ncopy; ++k)
+    for (int x = 0; x < kRows; ++x) {
+      uint32_t* row = out.data() + (size_t)k * (L.copy + 4 * G) + (size_t)x * L.stride;
       for (int z = 0; z < G; ++z)
         for (int q = 0; q < Q; ++q) {
           const uint16_t lo = (uint16_t)e_of(x, z * Q + q + 1);
           const uint16_t hi = (uint16_t)e_of(x, (z + G) * Q + q + 1);
-          out[(size_t)k * (copy + 4 * G) + (size_t)x * stride + word_index(z, q)] =
-              (uint32_t)lo | ((uint32_t)hi << 16);
+          const uint32_t v = (uint32_t)lo | ((uint32_t)hi << 16);
+          if (q < L.n4 * 4) {
+            row[(q / 4) * 4 * G + z * 4 + (q % 4)] = v;
+          } else if (L.has2 && q < L.n4 * 4 + 2) {
+            for (int j = 0; j < L.nc2; ++j) row[L.b2 + j * 2 * G + z * 2 + (q - L.n4 * 4)] = v;
+          } else {
+            for (int j = 0; j < L.nc1; ++j) row[L.b1 + j * G + z] = v;
+          }
         }
+    }
   return out;
 }
 

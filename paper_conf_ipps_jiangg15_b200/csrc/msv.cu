@@ -20,15 +20,18 @@ const void* msv_fast_ptr_g32(int q);
 
 int msv_q_max(int G) { return G == 32 ? 40 : 32; }
 
-int msv_table_words(int G, int Q) {
-  switch (G) {
-    case 4: {
-      const int stride = (Q * 4 + 31) / 32 * 32, copy = kRows * stride;
-      return ((2 * copy + 16) + 3) / 4 * 4;
-    }
-    default: return kRows * Q * G;
-  }
+int msv_table_words(int G, int Q) { return MsvLayoutRT(G, Q).words; }
+
+template <int G, int Q>
+constexpr bool msv_layout_agrees() {
+  constexpr MsvLayoutRT r(G, Q);
+  using Lt = MsvLayout<G, Q>;
+  return r.words == Lt::WORDS && r.stride == Lt::STRIDE && r.b2 == Lt::B2 && r.b1 == Lt::B1;
 }
+static_assert(msv_layout_agrees<4, 9>() && msv_layout_agrees<4, 10>() && msv_layout_agrees<8, 13>() &&
+              msv_layout_agrees<8, 26>() && msv_layout_agrees<8, 7>() && msv_layout_agrees<16, 13>() &&
+              msv_layout_agrees<16, 15>() && msv_layout_agrees<16, 18>() && msv_layout_agrees<32, 7>() &&
+              msv_layout_agrees<32, 25>(), "MsvLayoutRT != MsvLayout");
 
 static const void* msv_fast_ptr(int G, int Q) {
   switch (G) {

@@ -44,10 +44,22 @@ struct Chunks {
 // groups share a quarter-warp's LDS.128 wavefront while reading different residue rows; they
 // get their own copy of the table, shifted by 16*G bytes inside the 128-byte bank period
 // (row stride a multiple of 128 B), so their 16*G-byte chunks never share a bank.
+// For G = 8 / 16 the 4-word chunks are one quarter-warp's 128 B and never conflict, but the
+// remainder chunks (2 words per lane: LDS.64, split per half-warp; 1 word: LDS.32, whole warp)
+// are read by 2 or 4 groups of different residue rows in one wavefront: each row holds
+// 32 / (G * w) copies of such a chunk, copy j at bank offset j * G * w, and group grp reads copy
+// grp % NC -- conflict-free with the row stride a multiple of 32 words (it was 3.8% of the
+// config-3 kernel's shared-memory wavefronts, profiles/ncu_full_r02n.md).
 template <int G, int Q>
 struct MsvLayout {
+  using C = Chunks<Q>;
   static constexpr int NCOPY = G < 8 ? 8 / G : 1;
-  static constexpr int STRIDE = NCOPY > 1 ? (Q * G + 31) / 32 * 32 : Q * G;     // words per row
+  static constexpr int NC2 = G == 8 ? 2 : 1;                                    // copies of the 2-word chunk
+  static constexpr int NC1 = G == 8 ? 4 : (G == 16 ? 2 : 1);                    // copies of the 1-word chunk
+  static constexpr int B2 = C::n4 * 4 * G;                                      // 2-word chunk (copy 0)
+  static constexpr int B1 = B2 + (C::has2 ? 2 * G * NC2 : 0);                   // 1-word chunk (copy 0)
+  static constexpr int ROWW = B1 + (C::has1 ? G * NC1 : 0);
+  static constexpr int STRIDE = NCOPY > 1 ? (ROWW + 31) / 32 * 32 : ROWW;       // words per row
   static constexpr int COPY = kRows * STRIDE;                                   // words per copy
   static constexpr int WORDS = ((NCOPY * COPY + (NCOPY - 1) * 4 * G) + 3) / 4 * 4;
   __host__ __device__ static constexpr int base(int grp) { return (grp % NCOPY) * (COPY + 4 * G); }
@@ -74,6 +86,29 @@ __device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z
   }
 }
 
+// load_row in the MSV layout (MsvLayout<G, Q>: remainder chunks in per-group copies)
+template <int G, int Q>
+__device__ __forceinline__ void load_row_msv(const uint32_t* __restrict__ row, int z, int grp, uint32_t (&e)[Q]) {
+  using C = Chunks<Q>;
+  using Lt = MsvLayout<G, Q>;
+#pragma unroll
+  for (int c = 0; c < C::n4; ++c) {
+    uint4 v = *reinterpret_cast<const uint4*>(row + c * 4 * G + z * 4);
+    e[4 * c + 0] = v.x;
+    e[4 * c + 1] = v.y;
+    e[4 * c + 2] = v.z;
+    e[4 * c + 3] = v.w;
+  }
+  if constexpr (C::has2) {
+    uint2 v = *reinterpret_cast<const uint2*>(row + Lt::B2 + (grp % Lt::NC2) * 2 * G + z * 2);
+    e[4 * C::n4 + 0] = v.x;
+    e[4 * C::n4 + 1] = v.y;
+  }
+  if constexpr (C::has1) {
+    e[Q - 1] = row[Lt::B1 + (grp % Lt::NC1) * G + z];
+  }
+}
+
 // Residue stream of one sequence: 16-byte quads of packed words (24 residues) fetched two
 // quads ahead, so the DRAM/L2 latency of the residue stream hides behind >= 24 DP rows even
 // for short models.  Words past the sequence are all-31 (pad rows).
@@ -97,6 +132,14 @@ struct ResStream {
     return r;
   }
 };
+
+// Q <= 8: vote once per 6-row word and replay the word on a crossing (MSV_WORD_VOTE builds),
+// instead of the branch-free pass + checked re-run every geometry uses by default
+#ifdef MSV_WORD_VOTE
+constexpr bool kMsvWordVote = true;
+#else
+constexpr bool kMsvWordVote = false;
+#endif
 
 __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
@@ -147,8 +190,9 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
   };
 
   const int nqmax = (Lmax + 23) / 24;
+  const int nwmax = (Lmax + 5) / 6;                     // rows stop at the group's last word
   // All rows of the batch.  CHECK: the per-row J->B / overflow vote and update (Alg 1 l.16-20)
-  // after every row; without it (Q > 8, first pass) the rows run branch-free.
+  // after every row; without it (the first pass) the rows run branch-free.
   auto run = [&](auto check_tag) {
    constexpr bool CHECK = decltype(check_tag)::value;
    ResStream rs;
@@ -157,6 +201,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
    uint4 w4 = rs.next(iq);
 #pragma unroll 1
    for (int k = 0; k < 4; ++k) {
+    if (iq * 4 + k >= nwmax) break;                     // warp-uniform (Lmax is lane 0's)
     const uint32_t w = w4.x;
     w4.x = w4.y;
     w4.y = w4.z;
@@ -164,7 +209,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
     // one DP row (Alg 1 l.11-20); `check`: per-row J->B / overflow vote
     auto row = [&](int x, bool check) {
       uint32_t e[Q];
-      load_row<G, Q>(sm + x * ROWW, z, e);
+      load_row_msv<G, Q>(sm + x * ROWW, z, grp, e);
       // diagonal carry from the previous virtual lane (value after its emission)
       uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
       c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
@@ -200,7 +245,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
         }
       }
     };
-    if constexpr (Q <= 8) {
+    if constexpr (kMsvWordVote && Q <= 8) {
       // short rows: vote once per word (6 rows).  R is a running max, so a threshold crossing
       // anywhere in the word shows at its end; then the word is replayed from a snapshot
       // with the per-row vote (exact, and rare: only hits).
@@ -225,15 +270,17 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
    }
   };
   reset();
-  if constexpr (Q <= 8) {
+  if constexpr (kMsvWordVote && Q <= 8) {
     run(std::true_type{});
   } else {
-    // Long rows: first the whole batch without the per-row update -- a branch per row pins t[]
-    // to fixed registers, and ptxas then copies all Q of them back after every row (26
-    // IMAD.MOV per row at Q = 26, a third of the kernel's instructions; 9.6% of the kernel's
-    // time, profiles/stage_nocheck_r02zh.jsonl).  With the threshold fixed and R a running max,
-    // that pass is exact unless some cell reached the J->B / overflow threshold; then (rare:
-    // about 0.2% of config-3 sequences) the batch is scored again with the per-row update.
+    // First the whole batch without the per-row update -- a branch per row pins t[] to fixed
+    // registers, and ptxas then copies all Q of them back after every row (26 IMAD.MOV per row
+    // at Q = 26, a third of the kernel's instructions; 9.6% of the kernel's time,
+    // profiles/stage_nocheck_r02zh.jsonl); for short rows the per-word vote and its register
+    // snapshot cost registers (74 at G = 16, Q = 4: three blocks per SM).  With the threshold
+    // fixed and R a running max, that pass is exact unless some cell reached the J->B /
+    // overflow threshold; then (rare: about 0.2% of config-3 sequences) the batch is scored
+    // again with the per-row update.
     run(std::false_type{});
     if (__any_sync(0xffffffffu, (__vadd2(R, thrv) & 0x80008000u) != 0u)) {
       reset();
@@ -289,7 +336,7 @@ __device__ __forceinline__ bool msv_chunk(const MsvArgs& a, const uint32_t* __re
     for (int j = 0; j < 6; ++j) {
       const int x = (w >> (5 * j)) & 31;
       uint32_t e[Q];
-      load_row<G, Q>(sm + x * ROWW, z, e);
+      load_row_msv<G, Q>(sm + x * ROWW, z, 0, e);
       uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
       c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
       c = __byte_perm(c, negpair, sel);
@@ -357,12 +404,20 @@ __device__ __forceinline__ void msv_fast_body(const MsvArgs& a) {
   }
   constexpr int NG = 32 / G;
   const long long first = (QL > 0 || a.skip_long) ? a.nlong : 0;
+  // the next batch is claimed before the current one is scored, so the atomic's round trip
+  // overlaps the rows instead of stalling the warp between batches
+  unsigned long long nb = 0;
+  if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
   for (;;) {
-    unsigned long long b = 0;
-    if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);
-    b = __shfl_sync(0xffffffffu, b, 0);
+    const unsigned long long b = __shfl_sync(0xffffffffu, nb, 0);
     if (first + (long long)b >= a.nseq) break;
+#ifndef MSV_NO_PREFETCH
+    if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
+#endif
     msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
+#ifdef MSV_NO_PREFETCH
+    if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
+#endif
   }
 }
 

@@ -318,12 +318,14 @@ __global__ void __launch_bounds__(128) vit_pair_kernel(const VitArgs a) {
     V.start(tr, z, mv, a.tbm_min, a.safe, valid, gbits);
 
     const int nqmax = (Lmax + 23) / 24;
+    const int nwmax = (Lmax + 5) / 6;                 // rows stop at the warp's last word
     ResStream rs;
     rs.init(wp, nw);
     for (int iq = 0; iq < nqmax; ++iq) {
       uint4 w4 = rs.next(iq);
 #pragma unroll 1
       for (int k = 0; k < 4; ++k) {
+        if (iq * 4 + k >= nwmax) break;               // warp-uniform (Lmax is the warp's max)
         const uint32_t w = w4.x;
         w4.x = w4.y;
         w4.y = w4.z;
