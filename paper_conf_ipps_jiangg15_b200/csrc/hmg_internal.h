@@ -24,10 +24,18 @@ constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
 // remainder chunks' copy 0 (b2, b1), their copy counts, and the table size in words (WORDS).
 // The host table builder (host.cu msv_table) and the launchers use this; msv.cu checks it
 // against the template for every instantiated geometry.
+#ifdef MSV_NO_BYTE
+constexpr bool kMsvByte = false;     // A/B builds: the 2-word remainder stays s16x2
+#else
+constexpr bool kMsvByte = true;
+#endif
+// byte: G = 8 / 16 with a 2-word remainder hold it as one word of four int8 emissions per lane
+// (32 / G copies, widened by PRMT; valid when msv_byte_exact holds, else the exact kernel runs).
 struct MsvLayoutRT {
-  int n4, has2, has1, nc2, nc1, b2, b1, roww, ncopy, stride, copy, words;
+  int n4, has2, has1, byte, nc2, nc1, b2, b1, roww, ncopy, stride, copy, words;
   __host__ __device__ constexpr MsvLayoutRT(int G, int Q)
-      : n4(Q / 4), has2(Q % 4 >= 2), has1(Q % 2), nc2(G == 8 ? 2 : 1), nc1(G == 8 ? 4 : (G == 16 ? 2 : 1)),
+      : n4(Q / 4), has2(Q % 4 >= 2), has1(Q % 2), byte(kMsvByte && (G == 8 || G == 16) && Q % 4 >= 2),
+        nc2(G == 8 ? 2 : 1), nc1(G == 8 ? 4 : (G == 16 ? 2 : 1)),
         b2(Q / 4 * 4 * G), b1(Q / 4 * 4 * G + (Q % 4 >= 2 ? 2 * G * (G == 8 ? 2 : 1) : 0)),
         roww(Q / 4 * 4 * G + (Q % 4 >= 2 ? 2 * G * (G == 8 ? 2 : 1) : 0) +
              (Q % 2 ? G * (G == 8 ? 4 : (G == 16 ? 2 : 1)) : 0)),
@@ -38,6 +46,13 @@ struct MsvLayoutRT {
     words = ((ncopy * copy + (ncopy - 1) * 4 * G) + 3) / 4 * 4;
   }
 };
+
+// int8 emissions (clamped at -128) are exact in the MSV fast kernel when every cell that takes an
+// emission is at most 128 above B': cells stay below the J->B threshold, at most
+// 3 + tjb + tbm (+ bias within a voting row) above B'.
+__host__ __device__ constexpr bool msv_byte_exact(int tjb_max, int tbm, int bias) {
+  return 3 + tjb_max + tbm + bias <= 128;
+}
 
 // ---------------------------------------------------------------- MSV kernel arguments
 

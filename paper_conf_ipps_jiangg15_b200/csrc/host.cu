@@ -265,6 +265,13 @@ std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
           const uint32_t v = (uint32_t)lo | ((uint32_t)hi << 16);
           if (q < L.n4 * 4) {
             row[(q / 4) * 4 * G + z * 4 + (q % 4)] = v;
+          } else if (L.byte && q < L.n4 * 4 + 2) {    // int8 pair: bytes 2 (q - 4 n4) (lo, hi)
+            auto b8 = [](int16_t x) { return (uint32_t)(uint8_t)(int8_t)std::max<int>(x, -128); };
+            const int sh = 16 * (q - L.n4 * 4);
+            for (int j = 0; j < 32 / G; ++j) {
+              uint32_t& w = row[L.b2 + j * G + z];
+              w |= (b8((int16_t)lo) | (b8((int16_t)hi) << 8)) << sh;
+            }
           } else if (L.has2 && q < L.n4 * 4 + 2) {
             for (int j = 0; j < L.nc2; ++j) row[L.b2 + j * 2 * G + z * 2 + (q - L.n4 * 4)] = v;
           } else {
@@ -447,6 +454,14 @@ hmg_status vit_thr_table(hmg_profile* p, const hmg_db* db, double F, const int32
   }, out);
 }
 
+// the fast MSV kernel scores this profile over this DB: its precondition (bias < 66 + tbm, set at
+// profile creation) and, for a geometry with the int8 remainder chunk, msv_byte_exact at the DB's
+// longest sequence; otherwise the exact kernel scores every sequence
+bool msv_fast_on(const hmg_profile* p, const hmg_db* db) {
+  if (!p->msv_fast || p->msv_Q <= 0) return false;
+  return !MsvLayoutRT(p->msv_G, p->msv_Q).byte || msv_byte_exact(tjb_of(std::max(db->Lmax, 0)), p->tbm, p->bias);
+}
+
 MsvArgs msv_args(const hmg_profile* p, const hmg_db* db) {
   MsvArgs a{};
   a.words = db->d_words;
@@ -498,7 +513,7 @@ hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st,
   }
   a.counter = ctr;
   const int nwarps_exact = 148 * 16;
-  if (p->msv_fast && p->msv_Q > 0) {
+  if (msv_fast_on(p, db)) {
     int ok = 0;
     if (mark0) mark(0, st);
     if ((e = launch_msv_fast(p->msv_G, p->msv_Q, a, st, &ok, pdl))) return cuda_status(e);
@@ -520,7 +535,7 @@ hmg_status run_msv_fast(const hmg_profile* p, const hmg_db* db, cudaStream_t st,
 hmg_status run_msv_redo(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
   cudaError_t e = cudaSuccess;
   const int64_t n = db->nseq;
-  if (p->msv_fast && p->msv_Q > 0) {
+  if (msv_fast_on(p, db)) {
     MsvArgs a = msv_args(p, db);
     a.raw = raw_sorted;
     const int nwarps_exact = 148 * 16;
@@ -547,7 +562,7 @@ hmg_status run_msv_long_chunks(const hmg_profile* p, const hmg_db* db, cudaStrea
 hmg_status run_msv(const hmg_profile* p, const hmg_db* db, cudaStream_t st, uint8_t* raw_sorted, Scratch& S) {
   int64_t nlong = -1;
   mark(0, st);
-  if (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 && db->nlong > 0 && !tune_int("NO_LONG_LANE", 0)) {
+  if (p->long_QV > 0 && msv_fast_on(p, db) && db->nlong > 0 && !tune_int("NO_LONG_LANE", 0)) {
     LongArgs la{};
     hmg_status s = run_msv_long_chunks(p, db, st, raw_sorted, S, &la);
     if (s != HMG_OK) return s;
@@ -1496,7 +1511,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     // pipeline long lane (long.cu): chunked MSV of the longest sequences on the whole GPU, then
     // their Viterbi filter on SMs held alone by pipe_long_vit_kernel while the main MSV kernel
     // (programmatic dependent launch) fills the other SMs
-    const int64_t nlong = (p->long_QV > 0 && p->msv_fast && p->msv_Q > 0 &&
+    const int64_t nlong = (p->long_QV > 0 && msv_fast_on(p, db) &&
                            (p->long_pair || (!p->vit_generic && p->vit_W == 0)) &&
                            !tune_int("NO_LONG_LANE", 0)) ? db->nlong : 0;
     uint8_t* owned = nullptr;
@@ -1558,7 +1573,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     // sequences), so the long lane's exclusive-SM Viterbi overlaps all of them
     cudaStream_t ms = st;
     cudaEvent_t ms_done = nullptr;
-    const bool overlap = h_image && p->msv_fast && p->msv_Q > 0;
+    const bool overlap = h_image && msv_fast_on(p, db);
     if (h_image && !overlap) {                      // exact-kernel profiles: plain upload first
       for (int q = 1; q < nparts; ++q)
         if ((e = cudaStreamWaitEvent(st, up_ev[q], 0))) return cuda_status(e);
@@ -1823,7 +1838,9 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
   std::vector<int> slow;
   for (int i = 0; i < nprof; ++i) {
     hmg_profile* p = const_cast<hmg_profile*>(profs[i]);
-    if (p->msv_fast && p->msv_Q > 0) idx.push_back(i);
+    // (the bucket geometry is chosen below: the int8-chunk bound is required of every fast profile)
+    if (p->msv_fast && p->msv_Q > 0 && msv_byte_exact(tjb_of(std::max(db->Lmax, 0)), p->tbm, p->bias))
+      idx.push_back(i);
     else slow.push_back(i);
   }
   std::stable_sort(idx.begin(), idx.end(), [&](int a, int b) { return profs[a]->M > profs[b]->M; });

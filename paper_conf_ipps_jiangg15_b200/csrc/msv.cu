@@ -26,7 +26,8 @@ template <int G, int Q>
 constexpr bool msv_layout_agrees() {
   constexpr MsvLayoutRT r(G, Q);
   using Lt = MsvLayout<G, Q>;
-  return r.words == Lt::WORDS && r.stride == Lt::STRIDE && r.b2 == Lt::B2 && r.b1 == Lt::B1;
+  return r.words == Lt::WORDS && r.stride == Lt::STRIDE && r.b2 == Lt::B2 && r.b1 == Lt::B1 &&
+         (r.byte != 0) == Lt::BYTE && (!Lt::BYTE || Lt::NCB * G == 2 * G * Lt::NC2);   // byte chunk fits the slot
 }
 static_assert(msv_layout_agrees<4, 9>() && msv_layout_agrees<4, 10>() && msv_layout_agrees<8, 13>() &&
               msv_layout_agrees<8, 26>() && msv_layout_agrees<8, 7>() && msv_layout_agrees<16, 13>() &&

@@ -50,9 +50,16 @@ struct Chunks {
 // 32 / (G * w) copies of such a chunk, copy j at bank offset j * G * w, and group grp reads copy
 // grp % NC -- conflict-free with the row stride a multiple of 32 words (it was 3.8% of the
 // config-3 kernel's shared-memory wavefronts, profiles/ncu_full_r02n.md).
+// With BYTE (G = 8 / 16 and a 2-word remainder) that chunk is one word per lane holding its two
+// registers as four int8 emissions (clamped at -128, exact under msv_byte_exact), in 32 / G
+// per-group copies: one conflict-free LDS.32 wavefront per warp instead of the LDS.64's two, for
+// two PRMT per lane-row on the ALU pipe, which has room (the kernel is bound by the shared-memory
+// wavefronts: L1 99.7% busy, ALU 78%, profiles/ncu_full_r02zk.md).
 template <int G, int Q>
 struct MsvLayout {
   using C = Chunks<Q>;
+  static constexpr bool BYTE = kMsvByte && (G == 8 || G == 16) && C::has2;
+  static constexpr int NCB = 32 / G;                                            // copies of the byte chunk
   static constexpr int NCOPY = G < 8 ? 8 / G : 1;
   static constexpr int NC2 = G == 8 ? 2 : 1;                                    // copies of the 2-word chunk
   static constexpr int NC1 = G == 8 ? 4 : (G == 16 ? 2 : 1);                    // copies of the 1-word chunk
@@ -86,6 +93,15 @@ __device__ __forceinline__ void load_row(const uint32_t* __restrict__ row, int z
   }
 }
 
+// PRMT in its default mode: a selector nibble with its top bit set replicates the sign of the byte
+// it names (__byte_perm uses only the low three bits of each nibble)
+template <uint32_t SEL>
+__device__ __forceinline__ uint32_t prmt_sext(uint32_t v) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(r) : "r"(v), "n"(SEL));
+  return r;
+}
+
 // load_row in the MSV layout (MsvLayout<G, Q>: remainder chunks in per-group copies)
 template <int G, int Q>
 __device__ __forceinline__ void load_row_msv(const uint32_t* __restrict__ row, int z, int grp, uint32_t (&e)[Q]) {
@@ -99,7 +115,11 @@ __device__ __forceinline__ void load_row_msv(const uint32_t* __restrict__ row, i
     e[4 * c + 2] = v.z;
     e[4 * c + 3] = v.w;
   }
-  if constexpr (C::has2) {
+  if constexpr (Lt::BYTE) {
+    const uint32_t v = row[Lt::B2 + (grp % Lt::NCB) * G + z];
+    e[4 * C::n4 + 0] = prmt_sext<0x9180u>(v);    // s16x2 (sext b0, sext b1)
+    e[4 * C::n4 + 1] = prmt_sext<0xB3A2u>(v);    // s16x2 (sext b2, sext b3)
+  } else if constexpr (C::has2) {
     uint2 v = *reinterpret_cast<const uint2*>(row + Lt::B2 + (grp % Lt::NC2) * 2 * G + z * 2);
     e[4 * C::n4 + 0] = v.x;
     e[4 * C::n4 + 1] = v.y;
@@ -133,13 +153,21 @@ struct ResStream {
   }
 };
 
-// Q <= 8: vote once per 6-row word and replay the word on a crossing (MSV_WORD_VOTE builds),
-// instead of the branch-free pass + checked re-run every geometry uses by default
-#ifdef MSV_WORD_VOTE
-constexpr bool kMsvWordVote = true;
+// Short rows (Q <= 8): vote once per 6-row word and replay the word on a crossing, instead of the
+// branch-free pass + checked re-run of the whole batch.  Whole-warp batches (G = 32: the long
+// sequences of hmg_msv's long queue and the long lane's sequential fallback) always do: a re-run
+// doubles the latency of a sequence that sets the kernel's tail (config 2: 3.10 -> 2.84 ms,
+// profiles/cmp_r02zl.jsonl) -- except the pipeline long lane's sequential fallback (long.cu), which
+// measured faster branch-free (config-3 MSV stage 5.21 -> 5.13 ms, cmp_r02zl / cmp_r02zm).
+// MSV_WORD_VOTE_ALL builds use it for every Q <= 8 geometry (measured equal, cmp_r02zm.jsonl).
+template <int G, int Q>
+constexpr bool msv_word_vote() {
+#ifdef MSV_WORD_VOTE_ALL
+  return Q <= 8;
 #else
-constexpr bool kMsvWordVote = false;
+  return G == 32 && Q <= 8;
 #endif
+}
 
 __device__ __forceinline__ int msv_thr(int xJ, int bias) {
   // smallest t-scale value at which xJ could change J->B (xJ >= 190) or overflow
@@ -150,7 +178,7 @@ __device__ __forceinline__ int msv_thr(int xJ, int bias) {
 
 // Score one batch of 32/G sequences (sorted indices s0 + group) with G lanes per
 // sequence and Q s16x2 registers per lane, profile table `sm` in shared memory.
-template <int G, int Q>
+template <int G, int Q, bool WV = msv_word_vote<G, Q>()>
 __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
                                          long long send) {
   // sm: the table as laid out by MsvLayout<G, Q>
@@ -245,7 +273,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
         }
       }
     };
-    if constexpr (kMsvWordVote && Q <= 8) {
+    if constexpr (WV) {
       // short rows: vote once per word (6 rows).  R is a running max, so a threshold crossing
       // anywhere in the word shows at its end; then the word is replayed from a snapshot
       // with the per-row vote (exact, and rare: only hits).
@@ -270,7 +298,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
    }
   };
   reset();
-  if constexpr (kMsvWordVote && Q <= 8) {
+  if constexpr (WV) {
     run(std::true_type{});
   } else {
     // First the whole batch without the per-row update -- a branch per row pins t[] to fixed
@@ -404,20 +432,14 @@ __device__ __forceinline__ void msv_fast_body(const MsvArgs& a) {
   }
   constexpr int NG = 32 / G;
   const long long first = (QL > 0 || a.skip_long) ? a.nlong : 0;
-  // the next batch is claimed before the current one is scored, so the atomic's round trip
-  // overlaps the rows instead of stalling the warp between batches
-  unsigned long long nb = 0;
-  if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
+  // (claiming the next batch before scoring the current one measured no difference,
+  //  profiles/cmp_r02zl.jsonl)
   for (;;) {
-    const unsigned long long b = __shfl_sync(0xffffffffu, nb, 0);
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(a.counter, (unsigned long long)NG);
+    b = __shfl_sync(0xffffffffu, b, 0);
     if (first + (long long)b >= a.nseq) break;
-#ifndef MSV_NO_PREFETCH
-    if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
-#endif
     msv_batch<G, Q>(a, sm, first + (long long)b, a.nseq);
-#ifdef MSV_NO_PREFETCH
-    if (lane == 0) nb = atomicAdd(a.counter, (unsigned long long)NG);
-#endif
   }
 }
 

@@ -138,6 +138,40 @@ def test_msv_high_scores_fast_path():
     assert (want == 255).sum() > 0 and (want >= 190).sum() > 0
 
 
+@pytest.mark.parametrize("M,G", [(400, 8), (100, 8), (200, 16), (60, 16)])
+@pytest.mark.parametrize("top", [8.0, 10.0, 10.6, 10.9, 11.2, 13.0])
+def test_msv_int8_remainder_bound(M, G, top, tune):
+    """Lane geometries whose 2-register remainder is read as int8 emissions (G = 8 / 16, Q % 4 in
+    {2, 3}): raising the profile's top score moves 3 + tjb(Lmax) + tbm + bias across 128 -- below it
+    the fast kernel with the clamped int8 chunk, above it the exact kernel -- with planted hits so the
+    J->B re-entry and overflow paths run on both sides (tjb(~3000) = 30: at M = 400, tbm = 49, the
+    bound is bias <= 46, i.e. top <= 10.6 nats; at M = 200 top <= 12).  Bit-exact against the oracle."""
+    tune("MSV_G", str(G))
+    rng = np.random.default_rng(int(M * 10 + top * 7))
+    prof = synth.make_profile(M, 4000 + M, stress=True)
+    msc = prof.msc.copy()
+    best = np.argmax(msc[:, :20], axis=1)
+    msc[np.arange(M), best] = np.maximum(msc[np.arange(M), best], 2.0)
+    msc[M // 3, best[M // 3]] = top                     # sets the bias byte
+    seqs = []
+    for i in range(120):
+        L = int(rng.integers(1, 900)) if i % 10 else int(rng.integers(2000, 3100))
+        d = synth.random_dsq(rng, L, 29 if i % 7 == 0 else 20)
+        if i % 4 == 0 and L > 8:
+            seg = best[: min(L, M)].astype(np.uint8)[: int(rng.integers(3, min(L, M) + 1))]
+            a = int(rng.integers(0, L - len(seg) + 1))
+            d[a:a + len(seg)] = seg
+        seqs.append(d)
+    dsq, off = _db_from(seqs)
+    got, p = _msv_gpu(msc, dsq, off)
+    q = p.quant()
+    assert q["msv_lanes"] == G and q["msv_regs"] % 4 >= 2     # the int8-remainder layout
+    om = oracle.MSVProfile(msc)
+    want = oracle.msv_db(om, dsq, off)
+    assert np.array_equal(got, want)
+    assert (want >= 190).sum() > 0                             # hits chain through J
+
+
 def test_msv_all_minus_inf_redo_path():
     """Gap-only sequences: every cell <= B', the fast kernel defers to the exact kernel."""
     prof = synth.make_profile(77, 5)

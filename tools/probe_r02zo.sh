@@ -1,0 +1,35 @@
+#!/bin/bash
+# (r02zn with the PRMT sign mode fixed) MSV int8 remainder chunk (G = 8 / 16, Q % 4 >= 2): parity (incl. the bound test), then the default
+# build against MSV_NO_BYTE on configs 3 and 1/5-shaped geometries, ncu of the config-3 MSV kernel.
+set -u
+TAG=${1:-r02zo}
+O=gpurun_out
+mkdir -p $O
+timeout 1500 python -m pytest tests/test_gpu_parity.py tests/test_gpu_batch.py tests/test_gpu_fuzz.py -q -x \
+  -k "msv or pipeline or fuzz or batch or config or vit" > $O/tests_msv_$TAG.log 2>&1
+run() {
+  local tag=$1
+  for c in "--config 3 --batch 0" "--config 2 --batch 64"; do
+    echo "build=$tag $c" >> $O/cmp_$TAG.jsonl
+    timeout 300 python bench.py $c --steps 10 --no-cpu-baseline --no-e2e --no-forward --no-configs \
+      >> $O/cmp_$TAG.jsonl 2>> $O/cmp_$TAG.err
+  done
+}
+run default
+HMG_NVCC_EXTRA=-DMSV_NO_BYTE python -c "from paper_conf_ipps_jiangg15_b200 import build; build.build(force=True)"
+run nobyte
+python -c "from paper_conf_ipps_jiangg15_b200 import build; build.build(force=True)"
+run default2
+for T in "" "--tune NO_LONG_LANE=1" "--tune PIPE_LONG_SMS=16"; do
+  echo "c5/0 tune=[$T]" >> $O/c5_$TAG.jsonl
+  timeout 300 python bench.py --config 5 --which 0 --nseq 1250000 --batch 0 --steps 10 --no-cpu-baseline --no-e2e \
+    --no-forward --no-configs $T >> $O/c5_$TAG.jsonl 2>> $O/c5_$TAG.err
+done
+B="python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-graph --no-configs --no-forward --batch 0"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:msv_fast -s 3 -c 1 \
+  -o $O/msv_fast_$TAG -f $B > $O/ncu_full_msv_fast_$TAG.log 2>&1
+python tools/ncu_summary.py $O/msv_fast_$TAG.ncu-rep > $O/ncu_full_$TAG.md 2>&1
+ncu -i $O/msv_fast_$TAG.ncu-rep --page source --csv --print-source sass > $O/src_msv_fast_$TAG.csv 2>/dev/null
+mkdir -p /tmp/ncu_reps_$TAG
+mv $O/*_$TAG.ncu-rep /tmp/ncu_reps_$TAG/ 2>/dev/null
+echo "done $TAG"
