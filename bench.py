@@ -264,7 +264,7 @@ def kernel_roofline(ev, key, cells, ms, p_int, ops_per_cell, label, lds_bound=Fa
     """Roofline of one kernel launch from its live time.  Two resources bound these kernels
     (DESIGN.md 4.2, 4.3c): the ALU pipe (DPX ops, 64 lanes/clk/SM) and the shared-memory data
     path (LDS, 37.1 TB/s measured).  `bound` names the one ncu shows busiest for the kernel
-    (lds_bound: the MSV kernel, L1 92% vs ALU 73%); `achieved` is ALGORITHMIC work per launch
+    (lds_bound: the MSV kernel, L1 99% vs ALU 84%, profiles/ncu_full_r02zo.md); `achieved` is ALGORITHMIC work per launch
     (design bytes or essential ops per cell x cells) / live time.  Both resources are reported,
     each with the measured counterpart from the committed ncu capture / SASS mix."""
     e = ev.get(key, {})
@@ -286,6 +286,9 @@ def kernel_roofline(ev, key, cells, ms, p_int, ops_per_cell, label, lds_bound=Fa
                "frac": round(la / ev["lds_peak_tbs"], 4), "bytes_per_cell": design,
                "measured_bytes_per_cell": e["lds_bytes_per_cell"],
                "measured_frac": round(lm / ev["lds_peak_tbs"], 4), "peak_source": ev.get("lds_peak_source")}
+        for k_src, k_dst in (("lds_bytes_per_cell_source", "measured_source"), ("lds_design_note", "note")):
+            if k_src in e:
+                lds[k_dst] = e[k_src]
     if lds_bound and lds:
         r = {"bound": "lds", "kernel": label, "achieved": lds["achieved"], "peak": lds["peak"], "unit": "TB/s",
              "frac": lds["frac"], "algorithmic_bytes_per_cell": lds["bytes_per_cell"], "lds": lds, "alu": a}

@@ -91,7 +91,7 @@ __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
       raw = Rmax > Bp ? max(Rmax - A.m.bias - 3, 0) : 254;
       if (lane == 0) A.m.raw[j] = (uint8_t)raw;
     } else {
-      raw = msv_batch<32, QL>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
+      raw = msv_batch<32, QL, false>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
     }
     if (lane == 0) A.owned[j] = raw != 254;
   }

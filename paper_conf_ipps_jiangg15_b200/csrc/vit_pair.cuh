@@ -135,19 +135,10 @@ struct VitPairLane {
     }
   }
 
-  __device__ __forceinline__ void row(const uint32_t* __restrict__ rrow, const uint32_t* __restrict__ tbm, int z,
-                                      unsigned gbits) {
-    const uint32_t sel = (z == 0) ? 0x1054u : 0x3210u;   // lane 0: low <- floor, high <- lane G-1 low
-    const int src = (z + G - 1) & (G - 1);
-    uint32_t e[Q];
-    load_row<G, Q>(rrow, z, e);
-    // diagonal carries: row i-1 at the last node of the previous virtual lane
-    uint32_t cM = __shfl_sync(0xffffffffu, Mc[Q - 1], src, G);
-    uint32_t cI = __shfl_sync(0xffffffffu, Ic[Q - 1], src, G);
-    uint32_t cD = __shfl_sync(0xffffffffu, Dc[Q - 1], src, G);
-    cM = __byte_perm(cM, 0u, sel);
-    cI = __byte_perm(cI, 0u, sel);
-    cD = __byte_perm(cD, 0u, sel);
+  // Alg 2 l.15-20 for one row from the diagonal carries (cM, cI, cD: row i-1 at the last node of the
+  // previous virtual lane): M, I, the running max R, and D with its in-lane D->D chain; returns the
+  // lane's outgoing D carry (D (+) tDD at its last node)
+  __device__ __forceinline__ uint32_t cells(const uint32_t (&e)[Q], uint32_t cM, uint32_t cI, uint32_t cD) {
     // M and I (Alg 2 l.15-16, emission per reading R15), descending: q-1 still holds row i-1
 #pragma unroll
     for (int q = Q - 1; q >= 0; --q) {
@@ -170,37 +161,83 @@ struct VitPairLane {
 #pragma unroll
     for (int q = 1; q < Q; ++q)
       Dc[q] = __viaddmax_s16x2(Dc[q - 1], tDD[q - 1], __viaddmax_s16x2_relu(Mc[q - 1], tMD[q - 1], tMD[q - 1]));
-    uint32_t cout =
-        __viaddmax_s16x2(Dc[Q - 1], tDD[Q - 1], __viaddmax_s16x2_relu(Mc[Q - 1], tMD[Q - 1], tMD[Q - 1]));
-    // hit / overflow / safe-bound vote (Alg 2 l.22-24 on the rows that need it)
-    const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
-    const unsigned bal = __ballot_sync(0xffffffffu, hit);
-    if (bal) {
-      uint32_t mm = R;
+    return __viaddmax_s16x2(Dc[Q - 1], tDD[Q - 1], __viaddmax_s16x2_relu(Mc[Q - 1], tMD[Q - 1], tMD[Q - 1]));
+  }
+
+  __device__ __forceinline__ bool hit_vote() const { return (__vadd2(R, thrv) & 0x80008000u) != 0u; }
+
+  // a row whose running max reached the threshold (ballot bal != 0): Alg 2 l.22-24 -- E->J, J->B,
+  // the floor raised and every cell re-based, or overflow / the s32 re-score
+  __device__ __forceinline__ void on_hit(unsigned bal, const uint32_t* __restrict__ tbm, int z, unsigned gbits,
+                                         uint32_t& cout) {
+    uint32_t mm = R;
 #pragma unroll
-      for (int o = G / 2; o >= 1; o >>= 1) mm = __vmaxs2(mm, __shfl_xor_sync(0xffffffffu, mm, o));
-      const int mp = max((int)(mm & 0xffffu), (int)(mm >> 16));
-      bool mine = (bal & gbits) != 0u && state == 0;
-      bool okv = true;
-      if (mine) {
-        if (mp > safe) {
-          state = 2;                                  // beyond the 16-bit window: s32 re-score
-        } else if (mp + F >= 32767) {
-          state = 1;                                  // reading R17: overflow -> +inf, pass
-        } else {
-          xJ = mp + F - 500;                          // E->J (and E->C: xC == xJ)
-          const int xB = max(xJ, kBaseW) + move;
-          const int Fn = max(-32768, min(32767, xB + tbm_min));
-          rebase(Fn - F, cout);
-          F = Fn;
-          okv = set_bk(tbm, z, xB);
-          set_thr(min(max(xJ, kBaseW) + 501, 32767));
-        }
+    for (int o = G / 2; o >= 1; o >>= 1) mm = __vmaxs2(mm, __shfl_xor_sync(0xffffffffu, mm, o));
+    const int mp = max((int)(mm & 0xffffu), (int)(mm >> 16));
+    bool mine = (bal & gbits) != 0u && state == 0;
+    bool okv = true;
+    if (mine) {
+      if (mp > safe) {
+        state = 2;                                  // beyond the 16-bit window: s32 re-score
+      } else if (mp + F >= 32767) {
+        state = 1;                                  // reading R17: overflow -> +inf, pass
+      } else {
+        xJ = mp + F - 500;                          // E->J (and E->C: xC == xJ)
+        const int xB = max(xJ, kBaseW) + move;
+        const int Fn = max(-32768, min(32767, xB + tbm_min));
+        rebase(Fn - F, cout);
+        F = Fn;
+        okv = set_bk(tbm, z, xB);
+        set_thr(min(max(xJ, kBaseW) + 501, 32767));
       }
-      const bool bad = (__ballot_sync(0xffffffffu, !okv) & gbits) != 0u;
-      if (mine && bad) state = 2;
-      if ((bal & gbits) && state) kill();
     }
+    const bool bad = (__ballot_sync(0xffffffffu, !okv) & gbits) != 0u;
+    if (mine && bad) state = 2;
+    if ((bal & gbits) && state) kill();
+  }
+
+  // Lazy-F across virtual lanes (l.25, Fig 7): passes while any carry improves (reading R19)
+  __device__ __forceinline__ void lazy(uint32_t cout, int src, uint32_t sel) {
+    for (;;) {
+      uint32_t cin = __shfl_sync(0xffffffffu, cout, src, G);
+      cin = __byte_perm(cin, 0u, sel);
+      bool imp = __vmaxs2(cin, Dc[0]) != Dc[0];
+      if (!__any_sync(0xffffffffu, imp)) break;
+      Dc[0] = __vmaxs2(Dc[0], cin);
+      constexpr int K0 = Q < 3 ? Q : 3;      // most D->D runs die within a few nodes
+#pragma unroll
+      for (int q = 1; q < K0; ++q) {
+        const uint32_t nd = __viaddmax_s16x2_relu(Dc[q - 1], tDD[q - 1], tDD[q - 1]);
+        imp = imp && (__vmaxs2(nd, Dc[q]) != Dc[q]);
+        Dc[q] = __vmaxs2(Dc[q], nd);
+      }
+      if (__any_sync(0xffffffffu, imp)) {
+#pragma unroll
+        for (int q = K0; q < Q; ++q) Dc[q] = __viaddmax_s16x2(Dc[q - 1], tDD[q - 1], Dc[q]);
+        cout = __viaddmax_s16x2(Dc[Q - 1], tDD[Q - 1], cout);
+      } else {
+        break;
+      }
+    }
+  }
+
+  __device__ __forceinline__ void row(const uint32_t* __restrict__ rrow, const uint32_t* __restrict__ tbm, int z,
+                                      unsigned gbits) {
+    const uint32_t sel = (z == 0) ? 0x1054u : 0x3210u;   // lane 0: low <- floor, high <- lane G-1 low
+    const int src = (z + G - 1) & (G - 1);
+    uint32_t e[Q];
+    load_row<G, Q>(rrow, z, e);
+    // diagonal carries: row i-1 at the last node of the previous virtual lane
+    uint32_t cM = __shfl_sync(0xffffffffu, Mc[Q - 1], src, G);
+    uint32_t cI = __shfl_sync(0xffffffffu, Ic[Q - 1], src, G);
+    uint32_t cD = __shfl_sync(0xffffffffu, Dc[Q - 1], src, G);
+    cM = __byte_perm(cM, 0u, sel);
+    cI = __byte_perm(cI, 0u, sel);
+    cD = __byte_perm(cD, 0u, sel);
+    uint32_t cout = cells(e, cM, cI, cD);
+    // hit / overflow / safe-bound vote (Alg 2 l.22-24 on the rows that need it)
+    const unsigned bal = __ballot_sync(0xffffffffu, hit_vote());
+    if (bal) on_hit(bal, tbm, z, gbits, cout);
     if constexpr (SCAN) {
       // inclusive max-plus scan of (carry out, tDD cost) over the lanes, both halves
       uint32_t c = cout, sm = bcost;
@@ -235,28 +272,7 @@ struct VitPairLane {
       }
       return;
     }
-    // Lazy-F across virtual lanes (l.25, Fig 7): passes while any carry improves (reading R19)
-    for (;;) {
-      uint32_t cin = __shfl_sync(0xffffffffu, cout, src, G);
-      cin = __byte_perm(cin, 0u, sel);
-      bool imp = __vmaxs2(cin, Dc[0]) != Dc[0];
-      if (!__any_sync(0xffffffffu, imp)) break;
-      Dc[0] = __vmaxs2(Dc[0], cin);
-      constexpr int K0 = Q < 3 ? Q : 3;      // most D->D runs die within a few nodes
-#pragma unroll
-      for (int q = 1; q < K0; ++q) {
-        const uint32_t nd = __viaddmax_s16x2_relu(Dc[q - 1], tDD[q - 1], tDD[q - 1]);
-        imp = imp && (__vmaxs2(nd, Dc[q]) != Dc[q]);
-        Dc[q] = __vmaxs2(Dc[q], nd);
-      }
-      if (__any_sync(0xffffffffu, imp)) {
-#pragma unroll
-        for (int q = K0; q < Q; ++q) Dc[q] = __viaddmax_s16x2(Dc[q - 1], tDD[q - 1], Dc[q]);
-        cout = __viaddmax_s16x2(Dc[Q - 1], tDD[Q - 1], cout);
-      } else {
-        break;
-      }
-    }
+    lazy(cout, src, sel);
   }
 
   // raw xC (== xJ) = max over rows of xE - 500; 32767 on overflow; kRedo (re-score) when the
