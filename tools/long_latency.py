@@ -26,5 +26,14 @@ for M in (100, 400, 500):
         torch.cuda.synchronize()
         ts.append(st["msv_kernel"])
     ms = min(ts[1:])
+    raw = torch.zeros(D.nseq, dtype=torch.uint8, device="cuda")
+    tm = []
+    for r in range(4):                       # MSV alone: chunked long-lane MSV (+ sequential fallback)
+        hmg.hmg_msv(P, D, raw)
+        st = hmg.hmg_stage_times()
+        torch.cuda.synchronize()
+        tm.append(st["msv_kernel"])
+    msv_ms = min(tm[1:])
     print(json.dumps({"M": M, "L": L, "msv_stage_ms": round(ms, 3), "cycles_per_row": round(ms * 1e-3 * 1.965e9 / L, 1),
+                      "msv_only_ms": round(msv_ms, 3), "msv_cycles_per_row": round(msv_ms * 1e-3 * 1.965e9 / L, 1),
                       "survivors": int(out["n_survivors"].item()), "long_lane": D.long_lane() if hasattr(D, "long_lane") else None}))
