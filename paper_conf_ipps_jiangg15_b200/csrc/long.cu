@@ -91,7 +91,14 @@ __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {
       raw = Rmax > Bp ? max(Rmax - A.m.bias - 3, 0) : 254;
       if (lane == 0) A.m.raw[j] = (uint8_t)raw;
     } else {
-      raw = msv_batch<32, QL, false>(A.m, smm, (long long)j, A.nlong);   // sequential whole-warp DP
+      // the chunk that called for this re-run saw a crossing, so a branch-free pass first would be
+      // wasted: short rows (QL <= 4) vote once per word (msv_batch<32, QL>), longer ones run the
+      // checked pass only -- the per-word vote's register snapshot costs 28-30 registers in this
+      // kernel (fewer resident chunk warps).  Measured (profiles/cmp_r02zt.jsonl, ms per step):
+      // checked 5.80 / 2.99 / 7.27 / 15.61, per-word vote 5.88 / 2.82 / 7.00 / 15.81 on configs
+      // 3 (QL = 7) / 2 (QL = 4) / 5 at M = 100 (QL = 2) / 5 at M = 500 (QL = 8)
+      if constexpr (QL <= 4) raw = msv_batch<32, QL>(A.m, smm, (long long)j, A.nlong);
+      else raw = msv_batch<32, QL, false, true>(A.m, smm, (long long)j, A.nlong);   // sequential DP
     }
     if (lane == 0) A.owned[j] = raw != 254;
   }
@@ -167,7 +174,11 @@ __global__ void __launch_bounds__(128) pipe_long_vpair_kernel(const LongArgs A) 
   const uint32_t* smv = reinterpret_cast<const uint32_t*>(smem4);
   const uint32_t* tr = reinterpret_cast<const uint32_t*>(A.v.tr);
   const int lane = threadIdx.x & 31;
+#ifdef LONG_SCAN
+  VitPairLane<32, Q, true> V;                    // A/B: max-plus scan Lazy-F (f1) in the long lane
+#else
   VitPairLane<32, Q> V;
+#endif
   V.load(tr, lane);
   for (;;) {
     unsigned long long b = 0;

@@ -157,8 +157,8 @@ struct ResStream {
 // branch-free pass + checked re-run of the whole batch.  Whole-warp batches (G = 32: the long
 // sequences of hmg_msv's long queue and the long lane's sequential fallback) always do: a re-run
 // doubles the latency of a sequence that sets the kernel's tail (config 2: 3.10 -> 2.84 ms,
-// profiles/cmp_r02zl.jsonl) -- except the pipeline long lane's sequential fallback (long.cu), which
-// measured faster branch-free (config-3 MSV stage 5.21 -> 5.13 ms, cmp_r02zl / cmp_r02zm).
+// profiles/cmp_r02zl.jsonl); the long lane's sequential fallback (long.cu) runs only the checked
+// pass (CHECKED below).
 // MSV_WORD_VOTE_ALL builds use it for every Q <= 8 geometry (measured equal, cmp_r02zm.jsonl).
 template <int G, int Q>
 constexpr bool msv_word_vote() {
@@ -178,7 +178,9 @@ __device__ __forceinline__ int msv_thr(int xJ, int bias) {
 
 // Score one batch of 32/G sequences (sorted indices s0 + group) with G lanes per
 // sequence and Q s16x2 registers per lane, profile table `sm` in shared memory.
-template <int G, int Q, bool WV = msv_word_vote<G, Q>()>
+// CHECKED: the caller knows a cell reaches the threshold (the long lane's sequential fallback after
+// a chunk crossed it): only the pass with the per-row update (no branch-free pass first)
+template <int G, int Q, bool WV = msv_word_vote<G, Q>(), bool CHECKED = false>
 __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __restrict__ sm, long long s0,
                                          long long send) {
   // sm: the table as laid out by MsvLayout<G, Q>
@@ -298,7 +300,7 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
    }
   };
   reset();
-  if constexpr (WV) {
+  if constexpr (WV || CHECKED) {
     run(std::true_type{});
   } else {
     // First the whole batch without the per-row update -- a branch per row pins t[] to fixed
