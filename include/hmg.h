@@ -271,7 +271,8 @@ hmg_status hmg_prepare_thresholds(const hmg_profile* p, double F1, double F2, in
  * Knobs (int): MSV_G, VIT_G, MSV_LLONG, NO_LONG_LANE, FWD_QMAX, FWD_W, FWD_S, VIT_CTA, VIT_CTA_W,
  * VIT_GENERIC, NO_VIT_PAIR, VIT_PAIR_G, VIT_PAIR_CTA, VIT_SCAN, VIT_PAIR_W, VIT_PAIR_SG,
  * VIT_CPAIR2, LONG_S32, PIPE_LLONG, PIPE_CHUNK, UPLOAD_PARTS, UPLOAD_FIRST_PERMILLE, UPLOAD_GROW,
- * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS, VIT_WIDE (0 off, 1 shared, 2 tensor memory).
+ * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS, VIT_WIDE (0 off, 1 shared, 2 tensor memory),
+ * LONG_PAIR_SMALL (0: models of <= 128 nodes keep the s32 long lane).
  * Geometry knobs take effect at profile / DB
  * creation, schedule knobs at the next call.  HMG_EINVAL for an unknown name. */
 hmg_status hmg_set_tuning(const char* name, int value);

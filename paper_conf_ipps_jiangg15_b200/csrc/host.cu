@@ -179,7 +179,7 @@ const char* const kTuneNames[] = {
     "MSV_G", "VIT_G", "MSV_LLONG", "NO_LONG_LANE", "FWD_QMAX", "FWD_W", "FWD_S", "VIT_CTA", "VIT_CTA_W",
     "VIT_GENERIC", "NO_VIT_PAIR", "VIT_PAIR_G", "VIT_PAIR_CTA", "VIT_SCAN", "VIT_PAIR_W", "VIT_PAIR_SG",
     "VIT_CPAIR2", "LONG_S32", "PIPE_LLONG", "PIPE_CHUNK", "UPLOAD_PARTS", "UPLOAD_FIRST_PERMILLE",
-    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS", "VIT_WIDE"};
+    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS", "VIT_WIDE", "LONG_PAIR_SMALL"};
 std::mutex g_tune_mu;
 std::map<std::string, int> g_tune;
 
@@ -1043,6 +1043,10 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
   // pipeline long lane: whole-warp Viterbi with the pair lane (the pair tables when G = 32, models
   // up to 1024 nodes) or the s32 latency lane (models up to 512 nodes)
   const bool lpair = p->pair_G == 32 && p->pair_W == 0 && !p->pair_wide && !tune_int("LONG_S32", 0);
+  // models whose pair kernel uses lane groups (M <= 128): the long lane gets pair tables of its own
+  // in the whole-warp geometry (G = 32, ceil(M / 64) registers)
+  const bool lpair_own = !lpair && p->pair_G > 0 && p->pair_G < 32 && !tune_int("LONG_S32", 0) &&
+                         tune_int("LONG_PAIR_SMALL", 1);
   if (st == HMG_OK && tsc && (lpair || M <= 512) && !tune_int("NO_LONG_LANE", 0)) {
     const int QL = long_msv_q(M);
     auto tm = msv_table(*p, 32, QL);
@@ -1050,6 +1054,17 @@ hmg_status hmg_profile_create(int M, const float* msc, const float* tsc, const h
     if (lpair) {
       if (st == HMG_OK) {
         p->long_QV = p->pair_Q;
+        p->long_pair = true;
+        p->long_QL = QL;
+      }
+    } else if (lpair_own) {
+      const int Q32 = (M + 63) / 64;
+      std::vector<uint32_t> r, t;
+      vit_pair_tables(*p, 32, Q32, &r, &t);
+      if (st == HMG_OK) st = upload(reinterpret_cast<uint32_t**>(&p->d_long_rsc), r.data(), r.size());
+      if (st == HMG_OK) st = upload(reinterpret_cast<uint32_t**>(&p->d_long_tr), t.data(), t.size());
+      if (st == HMG_OK) {
+        p->long_QV = Q32;
         p->long_pair = true;
         p->long_QL = QL;
       }
@@ -1598,8 +1613,10 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       la.v.len = db->d_len;
       la.v.nseq = n;
       la.v.move = db->d_move;
-      la.v.rsc = reinterpret_cast<const int16_t*>(p->long_pair ? (void*)p->d_pair_rsc : (void*)p->d_long_rsc);
-      la.v.tr = reinterpret_cast<const int32_t*>(p->long_pair ? (void*)p->d_pair_tr : (void*)p->d_long_tr);
+      // (pair lane: the pair kernel's tables when it runs whole warps, else the long lane's own)
+      const bool own = p->d_long_rsc != nullptr;
+      la.v.rsc = reinterpret_cast<const int16_t*>(p->long_pair && !own ? (void*)p->d_pair_rsc : (void*)p->d_long_rsc);
+      la.v.tr = reinterpret_cast<const int32_t*>(p->long_pair && !own ? (void*)p->d_pair_tr : (void*)p->d_long_tr);
       la.v.tbm_min = p->tbm_min;
       la.v.safe = 32767 - p->rmax;
       la.v.M = p->M;

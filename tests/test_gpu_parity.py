@@ -590,6 +590,7 @@ def test_vit_block_kernel_delete_chains(M, tune):
 
 
 @pytest.mark.parametrize("chunk,sms,M,lane", [(1032, "0", 120, "s32"), (60, "0", 120, "s32"),
+                                               (1032, "0", 100, "pair"), (60, "2", 64, "pair"),
                                                (1032, "2", 120, "s32"), (1032, "0", 300, "pair"),
                                                (60, "3", 300, "s32"), (1032, "0", 700, "pair"),
                                                (200, "2", 1000, "pair")])
@@ -597,7 +598,8 @@ def test_pipeline_long_lane(chunk, sms, M, lane, tune):
     """The pipeline long lane: sequences longer than max(1500, 8 x mean) get chunked MSV (rows
     from the empty state M rows early) and whole-warp Viterbi on SMs held alone (the s32 latency
     lane, or the s16x2 pair lane for models of 129..1024 nodes).  Strong planted hits in some
-    long sequences force the sequential fallback (a chunk sees a J->B row)."""
+    long sequences force the sequential fallback (a chunk sees a J->B row).  Models of <= 128
+    nodes ("pair" at M = 64 / 100) run the pair lane on tables of their own (G = 32)."""
     tune("PIPE_CHUNK", str(chunk))
     if sms != "0":
         tune("PIPE_LONG_SMS", sms)

@@ -1,12 +1,15 @@
 """Per-row latency of the pipeline long lane's Viterbi: one long sequence that passes MSV (F1 = 1),
 scored by hmg_pipeline (chunked MSV on the whole GPU, then the long-lane Viterbi on one warp).
-usage: python tools/long_latency.py [L]"""
+usage: python tools/long_latency.py [L] [KNOB=V ...]"""
 import os, sys, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 from paper_conf_ipps_jiangg15_b200 import build, hmg, synth
 build.build()
 L = int(sys.argv[1]) if len(sys.argv) > 1 else 30000
+for kv in sys.argv[2:]:                      # tuning knobs NAME=V (hmg_set_tuning)
+    k, v = kv.split("=")
+    hmg.set_tuning(k, int(v))
 rng = np.random.default_rng(0)
 for M in (100, 400, 500):
     prof = synth.make_profile(M, 1000 + M)
