@@ -174,11 +174,9 @@ __global__ void __launch_bounds__(128) pipe_long_vpair_kernel(const LongArgs A) 
   const uint32_t* smv = reinterpret_cast<const uint32_t*>(smem4);
   const uint32_t* tr = reinterpret_cast<const uint32_t*>(A.v.tr);
   const int lane = threadIdx.x & 31;
-#ifdef LONG_SCAN
-  VitPairLane<32, Q, true> V;                    // A/B: max-plus scan Lazy-F (f1) in the long lane
-#else
+  // (measured slower here: the max-plus scan Lazy-F, 387 -> 559 cycles per lone row at
+  //  M = 400, and a latency row form with the carries exchanged in the first Lazy-F round)
   VitPairLane<32, Q> V;
-#endif
   V.load(tr, lane);
   for (;;) {
     unsigned long long b = 0;
