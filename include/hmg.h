@@ -272,7 +272,7 @@ hmg_status hmg_prepare_thresholds(const hmg_profile* p, double F1, double F2, in
  * VIT_GENERIC, NO_VIT_PAIR, VIT_PAIR_G, VIT_PAIR_CTA, VIT_SCAN, VIT_PAIR_W, VIT_PAIR_SG,
  * VIT_CPAIR2, LONG_S32, PIPE_LLONG, PIPE_CHUNK, UPLOAD_PARTS, UPLOAD_FIRST_PERMILLE, UPLOAD_GROW,
  * PIPE_LONG_SMS, MSV_BATCH_PAD, MSV_BATCH_ROUNDS, VIT_WIDE (0 off, 1 shared, 2 tensor memory),
- * LONG_PAIR_SMALL (0: models of <= 128 nodes keep the s32 long lane).
+ * LONG_PAIR_SMALL (0: models of <= 128 nodes keep the s32 long lane), UPLOAD_MSV_STREAMS.
  * Geometry knobs take effect at profile / DB
  * creation, schedule knobs at the next call.  HMG_EINVAL for an unknown name. */
 hmg_status hmg_set_tuning(const char* name, int value);
@@ -301,11 +301,12 @@ hmg_status hmg_stage_counts(int64_t* counts);
 
 /* hmg_db_upload + hmg_pipeline with the upload overlapped: the packed image (host, pinned; from
  * hmg_db_image of this DB) is copied in length-ordered parts on a side stream (a first part of
- * 5% of the residues, then 5 parts of about equal residues; tuning knobs UPLOAD_PARTS /
+ * 5% of the residues, then 4 parts of about equal residues; tuning knobs UPLOAD_PARTS /
  * UPLOAD_FIRST_PERMILLE / UPLOAD_GROW, hmg_set_tuning), each part's landing recorded as an event;
- * one MSV launch per part on a second side stream waits for its part's event only (the long lane
- * starts after the first part), so the H2D of the later parts hides behind the filter of the
- * earlier ones.
+ * one MSV launch per part waits for its part's event only, the parts' launches rotating over two
+ * side streams (UPLOAD_MSV_STREAMS) so each starts on the SMs the previous one's tail frees (the
+ * long lane starts after the first part): the H2D of the later parts hides behind the filter of
+ * the earlier ones.
  * Outputs and results are hmg_pipeline's.  The image must stay valid until the call's work on
  * `stream` has completed. */
 hmg_status hmg_pipeline_upload(const hmg_profile* p, hmg_db* db, const uint32_t* image, double F1, double F2,

@@ -179,7 +179,8 @@ const char* const kTuneNames[] = {
     "MSV_G", "VIT_G", "MSV_LLONG", "NO_LONG_LANE", "FWD_QMAX", "FWD_W", "FWD_S", "VIT_CTA", "VIT_CTA_W",
     "VIT_GENERIC", "NO_VIT_PAIR", "VIT_PAIR_G", "VIT_PAIR_CTA", "VIT_SCAN", "VIT_PAIR_W", "VIT_PAIR_SG",
     "VIT_CPAIR2", "LONG_S32", "PIPE_LLONG", "PIPE_CHUNK", "UPLOAD_PARTS", "UPLOAD_FIRST_PERMILLE",
-    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS", "VIT_WIDE", "LONG_PAIR_SMALL"};
+    "UPLOAD_GROW", "PIPE_LONG_SMS", "MSV_BATCH_PAD", "MSV_BATCH_ROUNDS", "VIT_WIDE", "LONG_PAIR_SMALL",
+    "UPLOAD_MSV_STREAMS"};
 std::mutex g_tune_mu;
 std::map<std::string, int> g_tune;
 
@@ -1543,7 +1544,7 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     cudaStream_t cs = nullptr;
     SideJoin join(st);                              // every exit: side streams joined into st
     if (h_image) {
-      nparts = std::max(2, std::min(kUploadParts, tune_int("UPLOAD_PARTS", 6)));   // profiles/upload_parts_r01.jsonl
+      nparts = std::max(2, std::min(kUploadParts, tune_int("UPLOAD_PARTS", 5)));   // profiles/e2e_r02zza.jsonl
       // a small first part (the filter waits for it; later parts land faster than MSV consumes
       // them), then equal parts of the rest
       const int first_pm = tune_int("UPLOAD_FIRST_PERMILLE", 50);   // profiles/upload_parts_r01b.jsonl
@@ -1586,22 +1587,31 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
     }
     // the parts' MSV kernels run on a second side stream (they never read the long lane's
     // sequences), so the long lane's exclusive-SM Viterbi overlaps all of them
+    // consecutive parts' MSV kernels rotate over nms side streams, so a part's kernel starts on the
+    // SMs the previous part's tail frees (UPLOAD_MSV_STREAMS, 1..4)
+    constexpr int kMaxMsvStreams = 4;
     cudaStream_t ms = st;
-    cudaEvent_t ms_done = nullptr;
+    cudaStream_t mss[kMaxMsvStreams] = {st, st, st, st};
+    cudaEvent_t ms_done[kMaxMsvStreams] = {};
     const bool overlap = h_image && msv_fast_on(p, db);
+    const int nms = overlap ? std::max(1, std::min(kMaxMsvStreams, tune_int("UPLOAD_MSV_STREAMS", 2))) : 1;
     if (h_image && !overlap) {                      // exact-kernel profiles: plain upload first
       for (int q = 1; q < nparts; ++q)
         if ((e = cudaStreamWaitEvent(st, up_ev[q], 0))) return cuda_status(e);
     }
     if (overlap) {
-      ms = side_streams(db->device)[1];
-      join.add(ms);
       cudaEvent_t f2 = nullptr;
       if ((e = cudaEventCreateWithFlags(&f2, cudaEventDisableTiming))) return cuda_status(e);
-      if ((e = cudaEventRecord(f2, st)) || (e = cudaStreamWaitEvent(ms, f2, 0))) return cuda_status(e);
+      if ((e = cudaEventRecord(f2, st))) return cuda_status(e);
+      for (int k = 0; k < nms; ++k) {
+        mss[k] = side_streams(db->device)[1 + k];
+        join.add(mss[k]);
+        if ((e = cudaStreamWaitEvent(mss[k], f2, 0))) return cuda_status(e);
+        if ((e = cudaEventCreateWithFlags(&ms_done[k], cudaEventDisableTiming))) return cuda_status(e);
+        join.events.push_back(ms_done[k]);
+      }
       cudaEventDestroy(f2);
-      if ((e = cudaEventCreateWithFlags(&ms_done, cudaEventDisableTiming))) return cuda_status(e);
-      join.events.push_back(ms_done);
+      ms = mss[0];
     }
     mark(0, st);
     if (nlong > 0) {
@@ -1634,14 +1644,17 @@ static hmg_status pipeline_impl(const hmg_profile* pc, const hmg_db* db, double 
       if (s != HMG_OK) return s;
     } else {
       for (int q = 0; q < nparts; ++q) {          // MSV of each part once it has landed
-        if ((e = cudaStreamWaitEvent(ms, up_ev[q], 0))) return cuda_status(e);
+        cudaStream_t mq = mss[q % nms];
+        if ((e = cudaStreamWaitEvent(mq, up_ev[q], 0))) return cuda_status(e);
         const int64_t lo = std::max(bnd[q], nlong), hi = bnd[q + 1];
         if (hi > lo) {
-          s = run_msv_fast(p, db, ms, raw_sorted, S, lo, false, false, mctr + 2 * q, hi);
+          s = run_msv_fast(p, db, mq, raw_sorted, S, lo, false, false, mctr + 2 * q, hi);
           if (s != HMG_OK) return s;
         }
       }
-      if ((e = cudaEventRecord(ms_done, ms)) || (e = cudaStreamWaitEvent(st, ms_done, 0))) return cuda_status(e);
+      for (int k = 0; k < nms; ++k)
+        if ((e = cudaEventRecord(ms_done[k], mss[k])) || (e = cudaStreamWaitEvent(st, ms_done[k], 0)))
+          return cuda_status(e);
     }
     s = run_msv_redo(p, db, st, raw_sorted, S);
     if (s != HMG_OK) return s;

@@ -742,7 +742,7 @@ def test_vit_pair_maxplus_scan(M, tune):
 
 
 @pytest.mark.parametrize("cfg,sched", [(1, None), (3, None), (3, (12, 700)), (3, (2, 1500)),
-                                       (3, (6, 1000)), (1, (12, 1000))])
+                                       (3, (6, 1000)), (1, (12, 1000)), (3, (6, 1000, 2)), (3, (3, 1000, 2))])
 def test_pipeline_upload_overlapped_equals_pipeline(cfg, sched, tune):
     """hmg_pipeline_upload (packed image re-sent from pinned host memory in length-ordered parts,
     MSV per part as it lands, long lane alongside) gives hmg_pipeline's outputs exactly; the device
@@ -751,6 +751,8 @@ def test_pipeline_upload_overlapped_equals_pipeline(cfg, sched, tune):
     if sched is not None:
         tune("UPLOAD_PARTS", sched[0])
         tune("UPLOAD_GROW", sched[1])
+        if len(sched) > 2:
+            tune("UPLOAD_MSV_STREAMS", sched[2])     # parts' MSV kernels on two alternating streams
     prof, db = synth.config(cfg)
     dsq, off = db.materialize()
     ev = _calibrate(prof) if cfg == 1 else (-9.5, math.log(2), -9.0, math.log(2))
