@@ -29,6 +29,11 @@ constexpr bool kMsvByte = false;     // A/B builds: the 2-word remainder stays s
 #else
 constexpr bool kMsvByte = true;
 #endif
+#ifdef MSV_Q_PLUS1
+constexpr bool kMsvQPlus1 = true;    // A/B builds: 2GQ >= M + 1 (a successor cell for node M)
+#else
+constexpr bool kMsvQPlus1 = false;
+#endif
 // byte: G = 8 / 16 with a 2-word remainder hold it as one word of four int8 emissions per lane
 // (32 / G copies, widened by PRMT; valid when msv_byte_exact holds, else the exact kernel runs).
 struct MsvLayoutRT {

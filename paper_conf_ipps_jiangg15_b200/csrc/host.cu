@@ -220,12 +220,14 @@ void msv_geometry(int M, int* G, int* Q) {
   int g = M < 80 ? 4 : M <= 450 ? 8 : M <= 640 ? 16 : 32;
   const int o = tune_int("MSV_G", 0);
   if (o == 4 || o == 8 || o == 16 || o == 32) g = o;
-  // 2GQ >= M + 1: node M must have a (padding) successor cell, because the
-  // fast kernel records each cell's value in the cell it feeds (t_{i+1}[k+1]).
-  int q = (M + 2 * g) / (2 * g);
+  // 2GQ >= M: the fast kernel records each cell's value in the cell it feeds (t_{i+1}[k+1]); node
+  // M's, which no cell receives when 2GQ = M, enters the running max through the outgoing carry
+  // (msv.cuh).  (MSV_Q_PLUS1 builds: 2GQ >= M + 1, a padding successor cell.)
+  const int extra = kMsvQPlus1 ? 1 : 0;
+  int q = (M + extra + 2 * g - 1) / (2 * g);
   while (q > msv_q_max(g) && g < 32) {
     g *= 2;
-    q = (M + 2 * g) / (2 * g);
+    q = (M + extra + 2 * g - 1) / (2 * g);
   }
   *G = g;
   *Q = q <= msv_q_max(g) ? q : 0;   // 0: no register kernel, exact kernel only
@@ -264,10 +266,10 @@ std::vector<uint32_t> msv_table(const hmg_profile& p, int G, int Q) {
           const uint16_t lo = (uint16_t)e_of(x, z * Q + q + 1);
           const uint16_t hi = (uint16_t)e_of(x, (z + G) * Q + q + 1);
           const uint32_t v = (uint32_t)lo | ((uint32_t)hi << 16);
+          auto b8 = [](int16_t x) { return (uint32_t)(uint8_t)(int8_t)std::max<int>(x, -128); };
           if (q < L.n4 * 4) {
             row[(q / 4) * 4 * G + z * 4 + (q % 4)] = v;
           } else if (L.byte && q < L.n4 * 4 + 2) {    // int8 pair: bytes 2 (q - 4 n4) (lo, hi)
-            auto b8 = [](int16_t x) { return (uint32_t)(uint8_t)(int8_t)std::max<int>(x, -128); };
             const int sh = 16 * (q - L.n4 * 4);
             for (int j = 0; j < 32 / G; ++j) {
               uint32_t& w = row[L.b2 + j * G + z];
@@ -1886,7 +1888,7 @@ static hmg_status msv_batch_impl(const hmg_profile* const* profs, int nprof, con
     msv_geometry(profs[idx[j]]->M, &G, &Q);
     const int r0 = (int)rows.size();
     while (j < idx.size()) {
-      const int qj = (profs[idx[j]]->M + 2 * G) / (2 * G);
+      const int qj = (profs[idx[j]]->M + (kMsvQPlus1 ? 1 : 0) + 2 * G - 1) / (2 * G);
       if ((int)rows.size() > r0 && 100 * qj < (100 - pad_pct) * Q) break;
       rows.push_back(idx[j]);
       ++j;

@@ -32,7 +32,7 @@ namespace hmg {
 
 // whole-warp MSV registers that cover a model of up to 32*QV nodes (2*32*QL >= 32*QV + 1)
 // whole-warp MSV registers for a model of M nodes: 2 * 32 * QL >= M + 1
-int long_msv_q(int M) { return (M + 1 + 63) / 64; }
+int long_msv_q(int M) { return (M + (kMsvQPlus1 ? 1 : 0) + 63) / 64; }   // 2 x 32 x QL >= M (msv.cuh)
 
 template <int QL>
 __global__ void __launch_bounds__(256) pipe_long_msv_kernel(const LongArgs A) {

@@ -54,7 +54,9 @@ struct Chunks {
 // registers as four int8 emissions (clamped at -128, exact under msv_byte_exact), in 32 / G
 // per-group copies: one conflict-free LDS.32 wavefront per warp instead of the LDS.64's two, for
 // two PRMT per lane-row on the ALU pipe, which has room (the kernel is bound by the shared-memory
-// wavefronts: L1 99.7% busy, ALU 78%, profiles/ncu_full_r02zk.md).
+// wavefronts: L1 99.7% busy, ALU 78%, profiles/ncu_full_r02zk.md).  Also taking the last 4-register
+// chunk as int8 (one LDS.64) cut the wavefronts another 7.6% but moved the kernel onto the ALU pipe
+// (89%) and measured slower (config 3 5.77 -> 5.99 ms, config 2 2.88 -> 3.44; cmp_r02zzc.jsonl).
 template <int G, int Q>
 struct MsvLayout {
   using C = Chunks<Q>;
@@ -241,15 +243,18 @@ __device__ __forceinline__ int msv_batch(const MsvArgs& a, const uint32_t* __res
       uint32_t e[Q];
       load_row_msv<G, Q>(sm + x * ROWW, z, grp, e);
       // diagonal carry from the previous virtual lane (value after its emission)
-      uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
-      c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
+      const uint32_t co = __vadd2(t[Q - 1], e[Q - 1]);
+      uint32_t c = __shfl_sync(0xffffffffu, co, (z + G - 1) & (G - 1), G);
       c = __byte_perm(c, negpair, sel);
 #pragma unroll
       for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
       t[0] = __vmaxs2(c, B2);
+      // R also takes the outgoing carry co (this row's cells, the next lane's t[0] before the floor):
+      // the high half of lane G-1 is node M's cell when 2GQ = M, which no lane receives
 #pragma unroll
       for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
-      if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+      if constexpr (Q % 2) R = __vimax3_s16x2(R, t[Q - 1], co);
+      else R = __vmaxs2(R, co);
       if (!check) return;
       // does any cell of this row reach the J->B / overflow threshold?
       const bool hit = (__vadd2(R, thrv) & 0x80008000u) != 0u;
@@ -367,8 +372,8 @@ __device__ __forceinline__ bool msv_chunk(const MsvArgs& a, const uint32_t* __re
       const int x = (w >> (5 * j)) & 31;
       uint32_t e[Q];
       load_row_msv<G, Q>(sm + x * ROWW, z, 0, e);
-      uint32_t c = __vadd2(t[Q - 1], e[Q - 1]);
-      c = __shfl_sync(0xffffffffu, c, (z + G - 1) & (G - 1), G);
+      const uint32_t co = __vadd2(t[Q - 1], e[Q - 1]);
+      uint32_t c = __shfl_sync(0xffffffffu, co, (z + G - 1) & (G - 1), G);
       c = __byte_perm(c, negpair, sel);
 #pragma unroll
       for (int q = Q - 1; q >= 1; --q) t[q] = __viaddmax_s16x2(t[q - 1], e[q - 1], B2);
@@ -376,7 +381,8 @@ __device__ __forceinline__ bool msv_chunk(const MsvArgs& a, const uint32_t* __re
       if (counting) {
 #pragma unroll
         for (int q = 0; q + 1 < Q; q += 2) R = __vimax3_s16x2(R, t[q], t[q + 1]);
-        if constexpr (Q % 2) R = __vmaxs2(R, t[Q - 1]);
+        if constexpr (Q % 2) R = __vimax3_s16x2(R, t[Q - 1], co);     // co: as in msv_batch
+        else R = __vmaxs2(R, co);
         if (__any_sync(0xffffffffu, (__vadd2(R, thrv) & 0x80008000u) != 0u)) return false;
       }
     }
