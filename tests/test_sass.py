@@ -21,13 +21,13 @@ CUOBJDUMP = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
 
 # kernel (mangled) -> minimum static VIADDMNMX.S16x2 / VIMNMX3.S16x2 counts
 KERNELS = {
-    "_ZN3hmg18msv_fast_kernel_mbILi8ELi26ELi3EEEvNS_7MsvArgsE": (150, 60),      # config 3 MSV (M = 400)
+    "_ZN3hmg18msv_fast_kernel_mbILi8ELi25ELi3EEEvNS_7MsvArgsE": (150, 60),      # config 3 MSV (M = 400, Q = 25)
     "_ZN3hmg15msv_fast_kernelILi8ELi13EEEvNS_7MsvArgsE": (60, 30),             # config 2 MSV (M = 200)
     "_ZN3hmg15vit_pair_kernelILi32ELi7ELb0EEEvNS_7VitArgsE": (40, 3),           # config 3 Viterbi stage
     "_ZN3hmg17vit_cpair2_kernelILi16ELi2ELi0EEEvNS_7VitArgsE": (120, 5),        # two-warp Viterbi (M <= 2048)
     "_ZN3hmg15vit_wide_kernelILi32ELb1EEEvNS_7VitArgsE": (300, 10),            # config 4 Viterbi (M = 2048, TMEM)
     "_ZN3hmg15vit_wide_kernelILi20ELb0EEEvNS_7VitArgsE": (300, 10),            # 1024 < M <= 1280 (shared memory)
-    "_ZN3hmg19msv_multi_kernel_mbILi8ELi26ELi3EEEvNS_12MsvMultiArgsE": (100, 50),  # f4 batch MSV
+    "_ZN3hmg19msv_multi_kernel_mbILi8ELi25ELi3EEEvNS_12MsvMultiArgsE": (100, 50),  # f4 batch MSV
     "_ZN3hmg22pipe_long_vpair_kernelILi7EEEvNS_8LongArgsE": (40, 3),           # config 3 long lane
 }
 EMULATION = [re.compile(r"LOP3\.LUT.*0x7f7f7f7f"), re.compile(r"LOP3\.LUT.*0x80808080"),
