@@ -656,7 +656,16 @@ def main():
                                 "peak_source": "%s sm_max_mhz x %d SMs x %d FP32 lanes x 2 (FMA)"
                                                % (src, nsm, FP32_LANES_PER_CLK_SM),
                                 "note": "stage = Viterbi-pass compaction + Forward kernel on %d sequences "
-                                        "(latency-bound at this size; tools/fwd_bench.py for throughput)" % nf}}
+                                        "(latency-bound at this size: see throughput)" % nf}}
+        # the same kernel over every sequence of the DB (hmg_forward, no list): its throughput
+        # roofline, where the Fig 1 stage above is bounded by the row latency of its longest sequence
+        fall = torch.empty(n, dtype=torch.float32, device=dev)
+        t_all = timed_ms(lambda: hmg.hmg_forward(P, D, fall, stream=stream), stream, flush, 2)
+        a_all = FWD_FLOPS_PER_CELL * M * res_local / (t_all * 1e-3) / 1e12
+        forward["throughput"] = {"sequences": n, "residues": int(res_local), "ms": round(t_all, 3),
+                                 "gcups": round(M * res_local / (t_all * 1e-3) / 1e9, 1),
+                                 "achieved_tflops": round(a_all, 3), "frac": round(a_all / fp_peak, 4),
+                                 "note": "hmg_forward over every sequence of the workload (throughput mode)"}
 
     # ---------------------------------------------------------------- many-profile batch
     if args.batch > 0 and single:
