@@ -20,10 +20,6 @@ constexpr int kBaseW = 12000;   // Viterbi word base (reading R2)
 constexpr int16_t kNegE = -16384;   // "minus infinity" emission / carry of the s16x2 MSV lanes
 constexpr int kNegW = -32768;       // word -inf (Alg 2 l.9 P:674)
 
-// MsvLayout<G, Q> (msv.cuh) for run-time (G, Q): words per residue row (STRIDE), the offsets of the
-// remainder chunks' copy 0 (b2, b1), their copy counts, and the table size in words (WORDS).
-// The host table builder (host.cu msv_table) and the launchers use this; msv.cu checks it
-// against the template for every instantiated geometry.
 #ifdef MSV_NO_BYTE
 constexpr bool kMsvByte = false;     // A/B builds: the 2-word remainder stays s16x2
 #else
@@ -34,6 +30,10 @@ constexpr bool kMsvQPlus1 = true;    // A/B builds: 2GQ >= M + 1 (a successor ce
 #else
 constexpr bool kMsvQPlus1 = false;
 #endif
+// MsvLayout<G, Q> (msv.cuh) for run-time (G, Q): words per residue row (STRIDE), the offsets of the
+// remainder chunks' copy 0 (b2, b1), their copy counts, and the table size in words (WORDS).
+// The host table builder (host.cu msv_table) and the launchers use this; msv.cu checks it
+// against the template for every instantiated geometry.
 // byte: G = 8 / 16 with a 2-word remainder hold it as one word of four int8 emissions per lane
 // (32 / G copies, widened by PRMT; valid when msv_byte_exact holds, else the exact kernel runs).
 struct MsvLayoutRT {
