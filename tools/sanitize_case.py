@@ -11,7 +11,7 @@ lens = [int(x) for x in rng.integers(5, 300, size=120)] + [1700, 2100]   # two l
 dsq = np.concatenate([synth.random_dsq(rng, L, 29) for L in lens]).astype(np.uint8)
 off = np.zeros(len(lens) + 1, np.int64); np.cumsum(lens, out=off[1:])
 for M, env in ((60, {}), (300, {}), (700, {}), (1500, {}), (2048, {"VIT_CPAIR2": 23}), (3500, {}),
-               (90, {"VIT_CTA": 1})):
+               (90, {"VIT_CTA": 1}), (400, {}), (100, {}), (64, {}), (512, {"MSV_G": 16}), (2048, {})):
     for k, v in env.items():
         hmg.set_tuning(k, v)
     prof = synth.make_profile(M, M, dd=(1.0, 9.0))
@@ -58,3 +58,14 @@ ob = hmg.alloc_batch_outputs(len(Ps), D.nseq)
 hmg.hmg_pipeline_batch(Ps, D, F1=0.5, F2=0.5, **ob)
 torch.cuda.synchronize()
 print("batch ok", ob["n_survivors"].tolist())
+# overlapped upload (parts on two MSV streams) at the 2GQ = M and int8-remainder geometries
+for M in (400, 100):
+    prof = synth.make_profile(M, 90 + M)
+    P = hmg.Profile(prof.msc, prof.tsc, ev=(-9.0, 0.693, -9.0, 0.693))
+    D = hmg.Database(dsq, off)
+    img = torch.empty(D.packed_bytes // 4, dtype=torch.int32, pin_memory=True)
+    D.image(img)
+    out = hmg.alloc_outputs(D.nseq)
+    hmg.hmg_pipeline_upload(P, D, img, F1=0.5, F2=0.5, **out)
+    torch.cuda.synchronize()
+    print("upload M", M, "ok", int(out["n_survivors"].item()))
