@@ -122,6 +122,18 @@ bool fwd_geometry(int M, int* T, int* Q, int qmax) {
   if (32 * w * qmax < M) return false;
   int q = 2;
   while (32 * w * q < M) q *= 2;
+  // one warp: 12 / 13 / 14 nodes per thread where they fit below 16 (M = 257 ... 448: at M = 400,
+  // 13 nodes -- 416 cells a row -- instead of 512)
+#ifndef FWD_NO_Q13
+  if (w == 1 && q == 16 && qmax >= 16)
+#else
+  if (false)                                      // A/B builds: powers of two only
+#endif
+    for (int qq = 12; qq < 16; ++qq)
+      if (qq != 15 && 32 * qq >= M) {
+        q = qq;
+        break;
+      }
   *T = 32 * w;
   *Q = q;
   return true;
@@ -130,7 +142,8 @@ bool fwd_geometry(int M, int* T, int* Q, int qmax) {
 // Host tables (odds, float32) in the kernel's layouts.  msc: [M][29] nats, tsc: [M][8] nats.
 void fwd_tables(int M, int T, int Q, const float* msc, const float* tsc, std::vector<float>* etab,
                 std::vector<float>* tr, std::vector<float>* cst) {
-  const int V = Q >= 4 ? 4 : Q, C = Q / V, ROWF = T * Q, SEG = T < 32 ? T : 32;   // SEG: shuffle segment
+  const int V = Q % 4 == 0 ? 4 : (Q % 2 == 0 ? 2 : 1);   // FwdVec<Q>::V (forward.cuh)
+  const int C = Q / V, ROWF = T * Q, SEG = T < 32 ? T : 32;   // SEG: shuffle segment
   etab->assign((size_t)kRows * ROWF, 0.0f);
   for (int x = 0; x < kAlpha; ++x)
     for (int t = 0; t < T; ++t)

@@ -12,7 +12,9 @@ namespace hmg {
 constexpr float kFwdRescale = 1099511627776.0f;   // 2^40: E above this triggers a rescale
 
 
-template <int Q> struct FwdVec { static constexpr int V = Q >= 4 ? 4 : Q; };
+// floats per vector load of the emission row: 4 when Q is a multiple of 4, else 2, else 1 (the
+// one-warp geometries with 12..14 nodes per thread fit M = 385..448 without 16-node padding)
+template <int Q> struct FwdVec { static constexpr int V = Q % 4 == 0 ? 4 : (Q % 2 == 0 ? 2 : 1); };
 
 __device__ __forceinline__ void group_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
@@ -114,10 +116,13 @@ __global__ void __launch_bounds__((W == 1 ? GL : 32 * W) * S, 1) fwd_kernel(cons
           const float4* p4 = reinterpret_cast<const float4*>(er) + c * T + t;
           const float4 v = shared ? *p4 : __ldg(p4);
           e[4 * c] = v.x; e[4 * c + 1] = v.y; e[4 * c + 2] = v.z; e[4 * c + 3] = v.w;
-        } else {
+        } else if constexpr (V == 2) {
           const float2* p2 = reinterpret_cast<const float2*>(er) + c * T + t;
           const float2 v = shared ? *p2 : __ldg(p2);
           e[2 * c] = v.x; e[2 * c + 1] = v.y;
+        } else {
+          const float* p1 = er + c * T + t;
+          e[c] = shared ? *p1 : __ldg(p1);
         }
       }
     };

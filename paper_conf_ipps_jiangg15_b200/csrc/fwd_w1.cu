@@ -1,4 +1,4 @@
-// Instantiations of fwd_kernel<1, Q, S> for Q = 2, 4, 8, 16 and S = 2, 4, 8, 12, and of the
+// Instantiations of fwd_kernel<1, Q, S> for Q = 2, 4, 8, 12, 13, 14, 16 and S = 2, 4, 8, 12, and of the
 // sub-warp lane-group kernels fwd_kernel<1, Q, S, 8> (Q = 2, 4).
 #include "forward.cuh"
 
@@ -6,7 +6,7 @@ namespace hmg {
 namespace {
 template <int Q>
 const void* pick_s(int s) {
-  if (Q == 16 && 32 * 1 * s > 256) return nullptr;   // 16 nodes/thread need ~250 registers
+  if (Q >= 12 && 32 * 1 * s > 256) return nullptr;   // 12-16 nodes/thread need ~200-250 registers
   if (s == 2) return reinterpret_cast<const void*>(&fwd_kernel<1, Q, 2>);
   if (s == 4) return reinterpret_cast<const void*>(&fwd_kernel<1, Q, 4>);
   if (s == 8) return reinterpret_cast<const void*>(&fwd_kernel<1, Q, 8>);
@@ -38,6 +38,9 @@ const void* fwd_ptr_w1(int q, int s) {
     case 2: return pick_s<2>(s);
     case 4: return pick_s<4>(s);
     case 8: return pick_s<8>(s);
+    case 12: return pick_s<12>(s);
+    case 13: return pick_s<13>(s);
+    case 14: return pick_s<14>(s);
     case 16: return pick_s<16>(s);
   }
   return nullptr;
