@@ -169,11 +169,12 @@ def test_host_only_handles_rejected_by_compute_calls(L):
 
 def test_forward_geometry_host_only(L):
     """Forward kernel geometry: 8-lane groups up to M = 32, then the
-    fewest warps at 16 nodes per thread and the fewest nodes; unsupported above 4096 nodes."""
+    fewest warps at 16 nodes per thread and the fewest nodes (one warp: 12 / 13 / 14 before 16);
+    unsupported above 4096 nodes."""
     for M, (T, Qn) in {1: (8, 2), 16: (8, 2), 17: (8, 4), 32: (8, 4), 33: (32, 2), 64: (32, 2), 65: (32, 4),
-                       128: (32, 4), 129: (32, 8),
-                       256: (32, 8), 257: (32, 16), 400: (32, 16), 513: (64, 16), 1000: (64, 16), 2048: (128, 16),
-                       4096: (256, 16)}.items():
+                       128: (32, 4), 129: (32, 8), 256: (32, 8), 257: (32, 12), 384: (32, 12), 385: (32, 13),
+                       400: (32, 13), 416: (32, 13), 417: (32, 14), 448: (32, 14), 449: (32, 16), 512: (32, 16),
+                       513: (64, 16), 1000: (64, 16), 2048: (128, 16), 4096: (256, 16)}.items():
         p = hmg.Profile(np.zeros((M, 29), np.float32), np.full((M, 8), -1.0, np.float32), device=-1)
         q = p.quant()
         assert (q["fwd_lanes"], q["fwd_nodes"], q["fwd_warps"]) == (T, Qn, max(1, T // 32)), M
